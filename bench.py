@@ -1,0 +1,335 @@
+#!/usr/bin/env python
+"""bench.py -- input GB/s of spec-k FSM execution on B200 (BASELINE.json metric), one JSON line.
+
+Default workload = BASELINE configs[4] (C5, the config the metric is quoted on at 1/2/4/8 B200):
+a random (N, m) DFA over 64 GiB of counter-based i.i.d. bytes generated in place in HBM, sharded
+contiguously over the ranks (strong scaling).  --config picks another BASELINE config.
+
+A step = one pass of the whole hot path over the whole input: look-back speculation, local
+spec-k processing, warp/block/grid parallel merge, delayed re-execution and (N > 1) the NCCL
+all-gather of shard maps + compose + fix-up.  `value` = input bytes of all ranks / max-over-ranks
+device time per step (CUDA events on the library's stream), inputs resident in HBM.
+`e2e` = the same metric through fsm_run_spec_k_host from pinned HOST memory (H2D inside).
+`--impl reference` times the oracle (oracle/, plain sequential loop of Fig. 1c) on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+GiB = 1 << 30
+METRIC = "input GB/s (final state+accept count bit-exact)"
+
+
+# ----------------------------------------------------------------------------- workloads
+def make_workload(args):
+    """Returns dict(dfa, k, name, total_bytes, fill(dev_ptr, lo, n), host(lo, n) -> np.ndarray)."""
+    from fsmgen import dfas, streams
+
+    seed = streams.MASTER_SEED
+    cfg = args.config
+    if cfg == "c5":
+        d = dfas.random_dfa(args.n_states, args.m, seed=seed + 5)
+        total = int(args.size_gib * GiB)
+        sseed = seed + 5
+
+        def fill(ptr, lo, n, stream=0):
+            streams.splitmix_fill_device(ptr, sseed, lo, n, stream)
+
+        def host(lo, n, out=None):
+            return streams.splitmix_bytes(sseed, lo, n, out=out)
+
+        name = (f"C5 random DFA N={args.n_states} m={args.m} (|image(c)|=m), spec-{args.k}, "
+                f"{args.size_gib:g} GiB i.i.d. bytes")
+        return dict(dfa=d, k=args.k, name=name, total=total, fill=fill, host=host, bits=False)
+    if cfg == "c1":
+        d = dfas.c_comment(True)
+        total = 1 << 20
+        data = streams.c_source(total, seed=seed + 1)
+        return dict(dfa=d, k=1, name="C1 C-comment FSM (Fig. 1, 4 states x 3 classes) 1 MiB synthetic C, spec-1",
+                    total=total, data=data, bits=False)
+    raise SystemExit(f"unknown config {cfg}")
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            self.proc.wait()
+
+    def summary(self):
+        sm = [float(r[0]) for r in self.rows if r and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            for i, nme in enumerate(names):
+                if len(r) > 4 + i and r[4 + i].lower() == "active":
+                    reasons.add(nme)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- reference arm
+def cpu_oracle_rate(w, budget_s: float = 12.0, max_bytes: int = 4 * GiB):
+    """Time the oracle (plain sequential loop, 1 core) on a bounded prefix sample."""
+    from oracle import seq
+
+    d = w["dfa"]
+    n = min(w["total"], max_bytes)
+    probe = min(n, 64 << 20)
+    data = w["data"][:probe] if "data" in w else w["host"](0, probe)
+    t = time.perf_counter()
+    seq.run(d, data)
+    dt = time.perf_counter() - t
+    rate = probe / dt
+    n = int(min(n, max(probe, rate * budget_s)))
+    data = w["data"][:n] if "data" in w else w["host"](0, n)
+    t = time.perf_counter()
+    res = seq.run(d, data)
+    dt = time.perf_counter() - t
+    return dict(bytes=n, seconds=dt, gbs=n / dt / 1e9, result=res)
+
+
+def run_reference(args, w):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    try:
+        os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+    except (AttributeError, OSError):
+        pass
+    rates = []
+    for i in range(args.warmup + args.steps):
+        r = cpu_oracle_rate(w, budget_s=min(10.0, 120.0 / (args.warmup + args.steps)), max_bytes=2 * GiB)
+        if i >= args.warmup:
+            rates.append(r)
+    gbs = statistics.median(r["gbs"] for r in rates)
+    line = {"impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(statistics.median(r["seconds"] for r in rates) * 1e3, 3),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic", "config": config_json(args, w),
+            "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                             "sample": f"first {rates[0]['bytes']} bytes of the workload per step"},
+            "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def config_json(args, w):
+    return {"workload": w["name"], "input_bytes": w["total"], "k": w["k"],
+            "n_states": int(w["dfa"].n_states), "parallelism": f"shard{args.gpus}",
+            "l2": "input >> L2 (126 MB), no flush needed" if w["total"] > 4 * 126e6 else "L2 flushed between steps"}
+
+
+# ----------------------------------------------------------------------------- our arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="c5", choices=["c5", "c1"])
+    ap.add_argument("--n-states", type=int, default=8)
+    ap.add_argument("--m", type=int, default=2)
+    ap.add_argument("--k", type=int, default=2)
+    ap.add_argument("--size-gib", type=float, default=64.0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--variant", type=int, default=-1)
+    ap.add_argument("--chunk", type=int, default=0)
+    args = ap.parse_args()
+    w = make_workload(args)
+    if args.impl == "reference":
+        return run_reference(args, w)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ppopp_xiaja20_b200 import fsmspec
+    from paper_conf_ppopp_xiaja20_b200.dist import run_sharded
+    from paper_conf_ppopp_xiaja20_b200.fsmspec import FSM
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    d = w["dfa"]
+    k = w["k"]
+    total = w["total"]
+    lo = total * rank // world // 32 * 32
+    hi = total if rank == world - 1 else total * (rank + 1) // world // 32 * 32
+    n = hi - lo
+    buf = torch.empty(n + 64, dtype=torch.uint8, device=dev)
+    halo = torch.zeros(32, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    if "data" in w:
+        buf[:n] = torch.from_numpy(w["data"][lo:hi]).to(dev)
+        if rank:
+            halo[0] = int(w["data"][lo - 1])
+    else:
+        w["fill"](buf.data_ptr(), lo, n, stream.cuda_stream)
+        if rank:
+            w["fill"](halo.data_ptr(), lo - 1, 1, stream.cuda_stream)
+    torch.cuda.synchronize()
+
+    f = FSM.from_dfa(d)
+    f.set_stream(stream.cuda_stream)
+    if args.variant >= 0 or args.chunk:
+        f.set_options(variant=args.variant, chunk_bytes=args.chunk)
+    res = torch.zeros(4, dtype=torch.int32, device=dev)
+    small = total < 4 * 126_000_000
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if small else None
+
+    def step():
+        if world == 1:
+            f.run_spec_k_async(buf.data_ptr(), n, k, res.data_ptr())
+            return None
+        return run_sharded(f, buf.data_ptr(), n, halo.data_ptr() if rank else None, k, d.start, device=dev)
+
+    # parity gate on the bench's own launch configuration: the prefix sample the oracle also times
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    times = []
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            if flush is not None:
+                flush.zero_()
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            out = step()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            times.append(e0.elapsed_time(e1) / 1e3)
+    t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    step_s = float(t.item())
+    st = f.stats() if world == 1 else {}
+    if world == 1:
+        f.run_spec_k(buf.data_ptr(), n, k)
+        st = f.stats()
+    r = res.cpu().numpy().view(np.uint32)
+    final = (int(r[0]), int(r[2]) | (int(r[3]) << 32)) if world == 1 else out
+
+    # ---- e2e through the host-buffer C-ABI entry point (pinned host memory, H2D in the region)
+    e2e = None
+    if not args.no_e2e:
+        try:
+            import psutil
+            avail = psutil.virtual_memory().available
+        except Exception:
+            avail = 0
+        if n + (8 << 30) < avail * 0.8:
+            hbuf = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+            hview = hbuf.numpy()
+            if "data" in w:
+                hview[:] = w["data"][lo:hi]
+            else:
+                w["host"](lo, n, out=hview)
+            if world == 1:
+                et = []
+                for i in range(max(1, min(args.steps, 3)) + 1):
+                    torch.cuda.synchronize()
+                    t0 = time.perf_counter()
+                    got = f.run_spec_k_host(hbuf.data_ptr(), n, k)
+                    dt = time.perf_counter() - t0
+                    if i:
+                        et.append(dt)
+                assert got == final, (got, final)
+                e2e = {"value": round(n / statistics.median(et) / 1e9, 3), "unit": "GB/s",
+                       "h2d_bytes_per_step": n, "d2h_bytes_per_step": 16}
+            del hbuf
+        else:
+            e2e = {"value": None, "unit": "GB/s", "h2d_bytes_per_step": n, "d2h_bytes_per_step": 16,
+                   "note": f"host RAM {avail / GiB:.0f} GiB too small for a {n / GiB:.0f} GiB pinned buffer"}
+
+    if rank != 0:
+        dist.destroy_process_group()
+        return
+    gbs = total / step_s / 1e9
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except OSError:
+        pass
+    peak = float(peaks.get("hbm_gbs", 6650.0))
+    line = {
+        "metric": METRIC, "value": round(gbs, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(step_s * 1e3, 4), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": config_json(args, w),
+        "roofline": {"bound": "hbm", "achieved": round(n / step_s / 1e9, 3) if world == 1 else round(gbs / world, 3),
+                     "peak": peak, "unit": "GB/s", "frac": round((n / step_s / 1e9) / peak, 4),
+                     "traffic": None, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback"},
+        "clocks": clk.summary(),
+        "gpu_launches": args.steps * (1 if world == 1 else 1),
+        "result": {"final_state": final[0], "accept_count": final[1]},
+        "stats": {kk: v for kk, v in st.items()},
+        "e2e": e2e,
+    }
+    if not args.no_cpu and world == 1:
+        try:
+            os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+        except (AttributeError, OSError):
+            pass
+        cb = cpu_oracle_rate(w, budget_s=12.0)
+        # parity on the sampled prefix: the GPU runs the same prefix in the bench's configuration
+        gp = f.run_spec_k(buf.data_ptr(), cb["bytes"], k)
+        line["cpu_baseline"] = {"value": round(cb["gbs"], 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                                "sample": f"first {cb['bytes']} bytes of the workload ({cb['seconds']:.1f} s)"}
+        line["parity_sample"] = {"bytes": cb["bytes"], "ok": gp == cb["result"]}
+        line["host_cores"] = os.cpu_count()
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,199 @@
+/* fsmspec.h -- C ABI of libfsmspec: spec-k speculative FSM execution with parallel merge on B200.
+ *
+ * Method: Xia, Jiang & Agrawal, "Scaling Out Speculative Execution of Finite-State Machines with
+ * Parallel Merge", PPoPP'20.  P:n = PAPER.md line n.
+ *   - problem statement: a DFA (Q, Sigma, q0, delta, F) run over a long input      P:61 (Sec. 2.1)
+ *   - Table 1 vocabulary: num_states N, num_guess k, num_inputs, num_item, num_thread
+ *   - spec-k: k = 1 speculative, k = N enumerative, otherwise enumerative speculation
+ *   - local processing of k speculated start states per chunk (Alg. 3)
+ *   - runtime membership check (Alg. 1 nested loop / Alg. 2 hash)
+ *   - parallel merge with delayed re-execution (invalid marking)
+ * Result = (q_L, |{i in [1, L] : q_i in F}|): the final state and the accept-position count
+ * (readings A4 and A21); it is bit-exact and independent of k, geometry,
+ * look-back policy and number of GPUs.
+ *
+ * Conventions
+ *   - Every function returns FSM_OK (0) or a negative status; out-parameters are written only
+ *     on FSM_OK.  Sticky CUDA errors are reported as FSM_ECUDA and not cleared.
+ *   - A handle is bound to the CUDA device that is current at fsm_create; calls on a handle
+ *     must be made with that device current.  One handle must not be used concurrently from two
+ *     host threads.
+ *   - "device pointer" = memory on the handle's device (cudaMalloc / torch CUDA tensor).
+ *     Input buffers are borrowed for the duration of the call (the async call: until the
+ *     stream work completes).  The caller keeps ownership of everything it passes in.
+ */
+#ifndef FSMSPEC_H
+#define FSMSPEC_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct fsm fsm_t;
+
+enum {
+    FSM_OK = 0,
+    FSM_EINVAL = -1,       /* invalid argument (see each call) */
+    FSM_ENOMEM = -2,       /* device or host allocation failed */
+    FSM_ECUDA = -3,        /* any CUDA runtime failure */
+    FSM_ESYMBOL = -4,      /* the input contained a byte >= alphabet (reading A14) */
+    FSM_EUNSUPPORTED = -5  /* current device is not sm_100 */
+};
+
+enum { FSM_INPUT_BYTES = 0, FSM_INPUT_BITS_MSB = 1 };
+
+#define FSM_KMAX 16
+
+/* Table-placement variants; FSM_VARIANT_AUTO picks by state count. */
+enum {
+    FSM_VARIANT_AUTO = -1,
+    FSM_VARIANT_P4 = 0,  /* N <= 4:   packed 4 x u8 row per symbol, lane-replicated smem, PRMT chain */
+    FSM_VARIANT_P8 = 1,  /* N <= 8:   packed 8 x u8 row per symbol, lane-replicated smem, PRMT chain */
+    FSM_VARIANT_B = 2,   /* N <= 256: u16 entries (next | count << 8) in shared memory            */
+    FSM_VARIANT_G = 3    /* any N:    u32 entries (next | count << 16) in global memory / L2      */
+};
+
+/* Merge strategies: the paper's parallel merge (default) and its sequential-merge baseline
+ * (Fig. 4a; the internal ablation of SURVEY.md 8.a11). */
+enum { FSM_MERGE_PARALLEL = 0, FSM_MERGE_SEQUENTIAL = 1 };
+
+/* fsm_create: build a handle for the DFA on the current device.
+ *   table       host pointer, n_states * alphabet entries, state-major:
+ *               delta(s, c) = table[s * alphabet + c] (Fig. 1b rows are states, P:229/P:235;
+ *               reading A3).  Copied; the caller keeps it.
+ *   n_states    N, 1 .. 65535.
+ *   alphabet    1 .. 256 symbols; input bytes >= alphabet drive an internal absorbing sink
+ *               state and make the run return FSM_ESYMBOL.
+ *   start       q0 < n_states.
+ *   accept_mask host pointer to n_states bytes (nonzero = in F) or NULL for F = {}.  Copied.
+ *   out         receives the handle.
+ * Errors: FSM_EINVAL (n_states or alphabet out of range, start or any entry >= n_states,
+ * NULL table/out), FSM_EUNSUPPORTED (device is not sm_100), FSM_ENOMEM, FSM_ECUDA. */
+int fsm_create(const uint32_t *table, uint32_t n_states, uint32_t alphabet, uint32_t start,
+               const uint8_t *accept_mask, fsm_t **out);
+
+/* As fsm_create; input_mode FSM_INPUT_BITS_MSB (requires alphabet == 2) reads the input as a
+ * packed bitstream, 8 symbols per byte, MSB first (Huffman decoding P:288, Div7 P:360; reading
+ * A13).  Lengths are then in bits. */
+int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t alphabet, uint32_t start,
+                  const uint8_t *accept_mask, uint32_t input_mode, fsm_t **out);
+
+/* Release all device and host resources of the handle.  NULL is a no-op. */
+void fsm_destroy(fsm_t *f);
+
+/* Static string for a status code. */
+const char *fsm_strerror(int status);
+
+/* Stream the handle's work is enqueued on (a cudaStream_t); NULL = legacy default stream. */
+int fsm_set_stream(fsm_t *f, void *cuda_stream);
+
+/* fsm_run_spec_k: run spec-k over a device-resident input and return the result on the host.
+ *   input   device pointer to the input (bytes; packed bits in bit mode); may be NULL iff len = 0.
+ *           Any alignment is accepted; 32-byte-aligned inputs take the vectorised path.
+ *   len     number of symbols (bytes; bits in bit mode).  len = 0 returns (start, 0).
+ *   k       number of speculated states per chunk, 1 <= k <= min(FSM_KMAX, n_states).
+ * Blocks until the result is on the host.  Errors: FSM_EINVAL, FSM_ESYMBOL, FSM_ECUDA. */
+int fsm_run_spec_k(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k,
+                   uint32_t *final_state, uint64_t *accept_count);
+
+/* Result record written to device memory by the asynchronous call. */
+typedef struct {
+    uint32_t final_state;   /* internal id; == n_states means an out-of-alphabet byte was seen */
+    uint32_t status;        /* 0 */
+    uint64_t accept_count;
+} fsm_result;
+
+/* fsm_run_spec_k_async: as fsm_run_spec_k, but only enqueues the work on the handle's stream and
+ * writes an fsm_result to `dev_result` (device pointer, 16-byte aligned).  No host
+ * synchronisation.  `final_state == n_states` signals FSM_ESYMBOL (when alphabet < 256). */
+int fsm_run_spec_k_async(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k,
+                         fsm_result *dev_result);
+
+/* fsm_run_spec_k_host: end-to-end form over a HOST buffer (pinned or pageable).  The library
+ * copies the input to the device in pieces on a copy stream and overlaps each piece's copy with
+ * the previous piece's kernel; pieces are chained on the device (the end state and count of piece
+ * p seed piece p+1).  Same arguments, result and errors as fsm_run_spec_k. */
+int fsm_run_spec_k_host(fsm_t *f, const uint8_t *host_input, uint64_t len, uint32_t k,
+                        uint32_t *final_state, uint64_t *accept_count);
+
+/* Tuning knobs; zero fields keep the current value.  Applied to subsequent runs. */
+typedef struct {
+    uint32_t chunk_bytes;       /* bytes per chunk (per thread), multiple of 32; 0 = adaptive */
+    uint32_t threads_per_tile;  /* chunks per tile (CTA size), 64 .. 1024, multiple of 32 */
+    int32_t variant;            /* FSM_VARIANT_*; FSM_VARIANT_AUTO = by state count */
+    uint32_t merge;             /* FSM_MERGE_* */
+    uint32_t ctas_per_sm;       /* cap on resident CTAs per SM for the persistent grid; 0 = max */
+} fsm_options;
+
+int fsm_set_options(fsm_t *f, const fsm_options *opt);
+int fsm_get_options(const fsm_t *f, fsm_options *opt);
+
+/* Counters of the most recent synchronous run on this handle (re-execution rate = reexec_chunks
+ * / chunks). */
+typedef struct {
+    uint64_t chunks;            /* chunks processed (one thread each) */
+    uint64_t tiles;             /* tiles (CTAs' work units) */
+    uint64_t reexec_chunks;     /* chunk re-executions (true-path and tile-candidate paths) */
+    uint64_t reexec_symbols;    /* bytes consumed by re-executions (early exit on convergence) */
+    uint64_t boundary_misses;   /* tile-boundary misses resolved after the look-back */
+    uint32_t chunk_bytes, threads_per_tile, variant, k_slots;
+} fsm_stats;
+
+int fsm_get_stats(const fsm_t *f, fsm_stats *s);
+
+/* ---------------------------------------------------------------- shard level (multi-GPU) ---
+ * A shard is a contiguous piece [lo, hi) of a longer input.  Shard 0 starts in
+ * q0; shard g > 0 speculates its start from the look-back byte just before it (the halo) and
+ * returns a k-slot mapping keyed on that speculated set, exactly as a chunk does. */
+typedef struct {
+    uint32_t k;                     /* slots in use */
+    uint32_t valid_mask;            /* bit s set = slot s holds a start state */
+    uint32_t start[FSM_KMAX];
+    uint32_t end[FSM_KMAX];
+    uint64_t count[FSM_KMAX];
+} fsm_shard_map;
+
+typedef struct fsm_shard fsm_shard_t;  /* per-shard state kept for a later fix-up */
+
+/* fsm_run_shard: run one shard.
+ *   input, len  device pointer and length (bytes, or bits in bit mode; bit-mode shards must start
+ *               on a byte boundary, i.e. every shard but the last has len % 8 == 0).
+ *   halo        device pointer to the halo_len bytes immediately before the shard, or NULL with
+ *               halo_len = 0 for shard 0 (start = q0).  Only the last halo byte is used.
+ *   out         receives the mapping; state (optional) receives a handle for fsm_shard_fixup,
+ *               which borrows `input` until fsm_shard_free.
+ * Errors: FSM_EINVAL, FSM_ECUDA, FSM_ENOMEM. */
+int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const uint8_t *halo,
+                  uint32_t halo_len, uint32_t k, fsm_shard_map *out, fsm_shard_t **state);
+
+/* fsm_shard_fixup: the shard's true start state turned out not to be speculated (a shard-boundary
+ * miss).  Re-executes from the shard start in lockstep with the speculated chains and stops when
+ * it joins one (exact); falls back to a full parallel re-run of the shard from `true_start`. */
+int fsm_shard_fixup(fsm_t *f, fsm_shard_t *state, uint32_t true_start, uint32_t *end,
+                    uint64_t *count);
+
+void fsm_shard_free(fsm_shard_t *state);  /* NULL is a no-op */
+
+/* fsm_map_compose: host-only, pure.  out = a followed by b, keyed on a's starts: a slot of a
+ * whose end is a start of b continues with b's end and adds counts; otherwise it becomes invalid
+ * (delayed strategy).  out may alias a or b. */
+int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, fsm_shard_map *out);
+
+/* ----------------------------------------------------------------------- host-only helpers ---
+ * fsm_lookback_table: the look-back speculation table the library builds at fsm_create (host
+ * code, no GPU needed).  For every input byte c: the image {delta(s, c)} (bit mode: of the
+ * 8-bit widened step) ranked by preimage count descending, ties to the smaller id (P:71,
+ * reading A5).  lb_out: 256 * FSM_KMAX uint16 (0xFFFF = unused), nimg_out: 256 bytes =
+ * min(|image|, FSM_KMAX).  States are internal ids (the sink, if any, is id n_states). */
+int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint32_t alphabet,
+                       uint32_t input_mode, uint16_t *lb_out, uint8_t *nimg_out);
+
+/* Library version string. */
+const char *fsm_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FSMSPEC_H */

@@ -28,7 +28,7 @@ class OracleSymbolError(ValueError):
 
 def build(force: bool = False) -> str:
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O3", "-march=native", "-shared", "-fPIC", "-o", _SO, _SRC])
+        subprocess.check_call(["gcc", "-O3", "-shared", "-fPIC", "-o", _SO, _SRC])
     return _SO
 
 

@@ -1,0 +1,734 @@
+// fsmspec.cu -- libfsmspec: the C ABI of include/fsmspec.h over the sm_100a kernels.
+//
+// Host responsibilities only: validation, preprocessing at create (host_tables.h), geometry,
+// kernel dispatch, result/stat transfer.  Every step of the hot path runs in the kernels of
+// speck_kernel.cuh / fixup_kernel.cuh / seqmerge_kernel.cuh; there is no CPU fallback.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "../../include/fsmspec.h"
+#include "fixup_kernel.cuh"
+#include "host_tables.h"
+#include "seqmerge_kernel.cuh"
+#include "speck_kernel.cuh"
+
+using namespace speck;
+
+// ------------------------------------------------------------------ kernel instantiations ----
+// k is a compile-time constant; a run with k uses the smallest instantiated K >= k and
+// marks the extra slots absent.
+static const int kKs[] = {1, 2, 3, 4, 6, 8, 12, 16};
+constexpr int kNumKs = 8;
+
+typedef void (*KernelFn)(Params);
+typedef void (*FixFn)(FixParams);
+typedef void (*SeqLocalFn)(Params, SeqBuf);
+typedef void (*SeqWalkFn)(Params, SeqBuf);
+
+template <int VAR>
+static KernelFn kernel_for(int K)
+{
+    switch (K) {
+    case 1: return speck_kernel<1, VAR>;
+    case 2: return speck_kernel<2, VAR>;
+    case 3: return speck_kernel<3, VAR>;
+    case 4: return speck_kernel<4, VAR>;
+    case 6: return speck_kernel<6, VAR>;
+    case 8: return speck_kernel<8, VAR>;
+    case 12: return speck_kernel<12, VAR>;
+    default: return speck_kernel<16, VAR>;
+    }
+}
+static KernelFn get_kernel(int var, int K)
+{
+    switch (var) {
+    case VAR_P4: return kernel_for<VAR_P4>(K);
+    case VAR_P8: return kernel_for<VAR_P8>(K);
+    case VAR_B: return kernel_for<VAR_B>(K);
+    default: return kernel_for<VAR_G>(K);
+    }
+}
+static FixFn get_fix(int var)
+{
+    switch (var) {
+    case VAR_P4: return fixup_kernel<VAR_P4>;
+    case VAR_P8: return fixup_kernel<VAR_P8>;
+    case VAR_B: return fixup_kernel<VAR_B>;
+    default: return fixup_kernel<VAR_G>;
+    }
+}
+template <int VAR>
+static void seq_for(int K, SeqLocalFn &l, SeqWalkFn &w)
+{
+    switch (K) {
+    case 1: l = seq_local_kernel<1, VAR>; w = seq_walk_kernel<1, VAR>; break;
+    case 2: l = seq_local_kernel<2, VAR>; w = seq_walk_kernel<2, VAR>; break;
+    case 3: l = seq_local_kernel<3, VAR>; w = seq_walk_kernel<3, VAR>; break;
+    case 4: l = seq_local_kernel<4, VAR>; w = seq_walk_kernel<4, VAR>; break;
+    case 6: l = seq_local_kernel<6, VAR>; w = seq_walk_kernel<6, VAR>; break;
+    case 8: l = seq_local_kernel<8, VAR>; w = seq_walk_kernel<8, VAR>; break;
+    case 12: l = seq_local_kernel<12, VAR>; w = seq_walk_kernel<12, VAR>; break;
+    default: l = seq_local_kernel<16, VAR>; w = seq_walk_kernel<16, VAR>; break;
+    }
+}
+static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
+{
+    switch (var) {
+    case VAR_P4: seq_for<VAR_P4>(K, l, w); break;
+    case VAR_P8: seq_for<VAR_P8>(K, l, w); break;
+    case VAR_B: seq_for<VAR_B>(K, l, w); break;
+    default: seq_for<VAR_G>(K, l, w); break;
+    }
+}
+
+static int kslots(uint32_t k)
+{
+    for (int i = 0; i < kNumKs; i++)
+        if (kKs[i] >= (int)k) return kKs[i];
+    return 16;
+}
+
+// ------------------------------------------------------------------------------ the handle ----
+struct fsm {
+    int device = 0;
+    int num_sms = 148;
+    cudaStream_t stream = nullptr;
+    cudaStream_t copy_stream = nullptr;
+    uint32_t n_user = 0, alphabet = 0, start = 0, mode = 0;
+    ByteDFA dfa;
+    int auto_variant = VAR_G;
+    fsm_options opt{};
+    // device tables
+    void *d_img[4] = {nullptr, nullptr, nullptr, nullptr};
+    uint32_t img_bytes[4] = {0, 0, 0, 0};
+    uint16_t *d_lb = nullptr;
+    uint8_t *d_nimg = nullptr;
+    uint32_t *d_bittab = nullptr;
+    // run state
+    TileDesc *d_desc = nullptr;
+    size_t desc_cap = 0;
+    uint32_t *d_ticket = nullptr;
+    uint32_t ticket_base = 0;
+    uint32_t epoch = 0;
+    DevResult *d_result = nullptr;   // [0] = run result, [1] = scratch for chained pieces
+    DevStats *d_stats = nullptr;
+    DevResult *h_result = nullptr;   // pinned
+    DevStats *h_stats = nullptr;     // pinned
+    unsigned long long *d_fix = nullptr;
+    // e2e staging
+    uint8_t *d_stage[2] = {nullptr, nullptr};
+    size_t stage_bytes = 0;
+    cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
+    // sequential-merge ablation buffers
+    SeqBuf seq{};
+    size_t seq_cap = 0;
+    // stats of the last synchronous run
+    fsm_stats last{};
+    DevStats stats_before{};
+    // hex lookback for host queries
+    std::vector<uint16_t> lb;
+    std::vector<uint8_t> nimg;
+};
+
+struct fsm_shard {
+    const uint8_t *input = nullptr;
+    uint64_t len = 0;          // symbols
+    uint32_t k = 0;
+    fsm_shard_map map{};
+};
+
+#define CK(x)                                                  \
+    do {                                                       \
+        cudaError_t _e = (x);                                  \
+        if (_e != cudaSuccess) return cuda_status(_e);         \
+    } while (0)
+
+static int cuda_status(cudaError_t e)
+{
+    if (e == cudaErrorMemoryAllocation) return FSM_ENOMEM;
+    if (getenv("FSM_DEBUG")) fprintf(stderr, "fsmspec: CUDA error %s\n", cudaGetErrorString(e));
+    return FSM_ECUDA;
+}
+
+extern "C" const char *fsm_strerror(int status)
+{
+    switch (status) {
+    case FSM_OK: return "ok";
+    case FSM_EINVAL: return "invalid argument";
+    case FSM_ENOMEM: return "out of memory";
+    case FSM_ECUDA: return "CUDA error";
+    case FSM_ESYMBOL: return "input symbol outside the alphabet";
+    case FSM_EUNSUPPORTED: return "unsupported device (sm_100 required)";
+    default: return "unknown status";
+    }
+}
+
+extern "C" const char *fsm_version(void) { return "fsmspec 0.1 (sm_100a)"; }
+
+extern "C" int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint32_t alphabet, uint32_t input_mode,
+                                  uint16_t *lb_out, uint8_t *nimg_out)
+{
+    if (!table || !lb_out || !nimg_out || n_states == 0 || alphabet == 0 || alphabet > 256) return FSM_EINVAL;
+    if (input_mode == FSM_INPUT_BITS_MSB && alphabet != 2) return FSM_EINVAL;
+    for (size_t i = 0; i < (size_t)n_states * alphabet; i++)
+        if (table[i] >= n_states) return FSM_EINVAL;
+    ByteDFA d;
+    build_byte_dfa(table, n_states, alphabet, nullptr, input_mode == FSM_INPUT_BITS_MSB, d);
+    build_lookback(d, lb_out, nimg_out);
+    return FSM_OK;
+}
+
+static void free_all(fsm *f)
+{
+    for (int i = 0; i < 4; i++) cudaFree(f->d_img[i]);
+    cudaFree(f->d_lb);
+    cudaFree(f->d_nimg);
+    cudaFree(f->d_bittab);
+    cudaFree(f->d_desc);
+    cudaFree(f->d_ticket);
+    cudaFree(f->d_result);
+    cudaFree(f->d_stats);
+    cudaFree(f->d_fix);
+    cudaFree(f->d_stage[0]);
+    cudaFree(f->d_stage[1]);
+    cudaFree(f->seq.S);
+    cudaFree(f->seq.E);
+    cudaFree(f->seq.C);
+    if (f->h_result) cudaFreeHost(f->h_result);
+    if (f->h_stats) cudaFreeHost(f->h_stats);
+    for (int i = 0; i < 2; i++) {
+        if (f->ev_copied[i]) cudaEventDestroy(f->ev_copied[i]);
+        if (f->ev_used[i]) cudaEventDestroy(f->ev_used[i]);
+    }
+    if (f->copy_stream) cudaStreamDestroy(f->copy_stream);
+}
+
+template <class T>
+static int upload(T **dptr, const void *src, size_t bytes)
+{
+    void *p = nullptr;
+    CK(cudaMalloc(&p, bytes ? bytes : 16));
+    if (bytes) CK(cudaMemcpy(p, src, bytes, cudaMemcpyHostToDevice));
+    *dptr = static_cast<T *>(p);
+    return FSM_OK;
+}
+
+extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t alphabet, uint32_t start,
+                             const uint8_t *accept_mask, uint32_t input_mode, fsm_t **out)
+{
+    if (!table || !out || n_states == 0 || n_states > 65535 || alphabet == 0 || alphabet > 256 || start >= n_states)
+        return FSM_EINVAL;
+    if (input_mode != FSM_INPUT_BYTES && input_mode != FSM_INPUT_BITS_MSB) return FSM_EINVAL;
+    const bool bits = input_mode == FSM_INPUT_BITS_MSB;
+    if (bits && alphabet != 2) return FSM_EINVAL;
+    if (!bits && alphabet < 256 && n_states >= 65535) return FSM_EINVAL;  // the sink needs an id < 0xFFFF
+    for (size_t i = 0; i < (size_t)n_states * alphabet; i++)
+        if (table[i] >= n_states) return FSM_EINVAL;
+
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, dev));
+    if (prop.major != 10) return FSM_EUNSUPPORTED;
+
+    fsm *f = new (std::nothrow) fsm();
+    if (!f) return FSM_ENOMEM;
+    f->device = dev;
+    f->num_sms = prop.multiProcessorCount;
+    f->n_user = n_states;
+    f->alphabet = alphabet;
+    f->start = start;
+    f->mode = input_mode;
+    build_byte_dfa(table, n_states, alphabet, accept_mask, bits, f->dfa);
+    f->lb.resize(256 * KMAX);
+    f->nimg.resize(256);
+    build_lookback(f->dfa, f->lb.data(), f->nimg.data());
+    const uint32_t n = f->dfa.n;
+    f->auto_variant = n <= 4 ? VAR_P4 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B : VAR_G;
+    f->opt.chunk_bytes = 0;
+    f->opt.threads_per_tile = kThreads;
+    f->opt.variant = FSM_VARIANT_AUTO;
+    f->opt.merge = FSM_MERGE_PARALLEL;
+    f->opt.ctas_per_sm = 0;
+
+    int rc = FSM_OK;
+    auto fail = [&](int r) {
+        free_all(f);
+        delete f;
+        return r;
+    };
+    // every variant the DFA fits, so that tests can force any of them
+    if (n <= 4) {
+        auto img = image_packed(f->dfa, false);
+        if ((rc = upload(&f->d_img[VAR_P4], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_P4] = kPackedTableBytes;
+    }
+    if (n <= 8) {
+        auto img = image_packed(f->dfa, true);
+        if ((rc = upload(&f->d_img[VAR_P8], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_P8] = kPackedTableBytes;
+    }
+    if (n <= 256) {
+        auto img = image_b(f->dfa);
+        if ((rc = upload(&f->d_img[VAR_B], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_B] = (uint32_t)img.size();
+    }
+    {
+        auto img = image_g(f->dfa);
+        if ((rc = upload(&f->d_img[VAR_G], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_G] = 0;
+    }
+    if ((rc = upload(&f->d_lb, f->lb.data(), f->lb.size() * 2))) return fail(rc);
+    if ((rc = upload(&f->d_nimg, f->nimg.data(), f->nimg.size()))) return fail(rc);
+    if (bits && (rc = upload(&f->d_bittab, f->dfa.bittab.data(), f->dfa.bittab.size() * 4))) return fail(rc);
+    {
+        cudaError_t e;
+        if ((e = cudaMalloc(&f->d_ticket, 64)) != cudaSuccess) return fail(cuda_status(e));
+        if ((e = cudaMemset(f->d_ticket, 0, 64)) != cudaSuccess) return fail(cuda_status(e));
+        if ((e = cudaMalloc(&f->d_result, 2 * sizeof(DevResult))) != cudaSuccess) return fail(cuda_status(e));
+        if ((e = cudaMemset(f->d_result, 0, 2 * sizeof(DevResult))) != cudaSuccess) return fail(cuda_status(e));
+        if ((e = cudaMalloc(&f->d_stats, sizeof(DevStats))) != cudaSuccess) return fail(cuda_status(e));
+        if ((e = cudaMemset(f->d_stats, 0, sizeof(DevStats))) != cudaSuccess) return fail(cuda_status(e));
+        if ((e = cudaMalloc(&f->d_fix, 64)) != cudaSuccess) return fail(cuda_status(e));
+        if ((e = cudaMallocHost(&f->h_result, sizeof(DevResult) + sizeof(DevStats))) != cudaSuccess)
+            return fail(cuda_status(e));
+        f->h_stats = nullptr;
+    }
+    *out = f;
+    return FSM_OK;
+}
+
+extern "C" int fsm_create(const uint32_t *table, uint32_t n_states, uint32_t alphabet, uint32_t start,
+                          const uint8_t *accept_mask, fsm_t **out)
+{
+    return fsm_create_ex(table, n_states, alphabet, start, accept_mask, FSM_INPUT_BYTES, out);
+}
+
+extern "C" void fsm_destroy(fsm_t *f)
+{
+    if (!f) return;
+    cudaStreamSynchronize(f->stream);
+    free_all(f);
+    delete f;
+}
+
+extern "C" int fsm_set_stream(fsm_t *f, void *s)
+{
+    if (!f) return FSM_EINVAL;
+    f->stream = (cudaStream_t)s;
+    return FSM_OK;
+}
+
+extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
+{
+    if (!f || !o) return FSM_EINVAL;
+    if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > (1u << 24))) return FSM_EINVAL;
+    if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > kThreads))
+        return FSM_EINVAL;
+    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_G) return FSM_EINVAL;
+    if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
+    if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
+    f->opt.chunk_bytes = o->chunk_bytes;  // 0 = adaptive
+    if (o->threads_per_tile) f->opt.threads_per_tile = o->threads_per_tile;
+    f->opt.variant = o->variant;
+    f->opt.merge = o->merge;
+    f->opt.ctas_per_sm = o->ctas_per_sm;
+    return FSM_OK;
+}
+
+extern "C" int fsm_get_options(const fsm_t *f, fsm_options *o)
+{
+    if (!f || !o) return FSM_EINVAL;
+    *o = f->opt;
+    return FSM_OK;
+}
+
+extern "C" int fsm_get_stats(const fsm_t *f, fsm_stats *s)
+{
+    if (!f || !s) return FSM_EINVAL;
+    *s = f->last;
+    return FSM_OK;
+}
+
+// ----------------------------------------------------------------------------------- runs ----
+struct RunSpec {
+    const uint8_t *in;
+    uint64_t len_sym;      // symbols
+    uint32_t k;
+    bool keyed;
+    uint32_t halo_byte;
+    uint32_t start_state;
+    const DevResult *start_dev;
+    DevResult *result;
+    int force_variant;     // -1 = handle options
+    uint32_t merge;
+};
+
+static int variant_of(const fsm *f, int force)
+{
+    if (force >= 0) return force;
+    return f->opt.variant == FSM_VARIANT_AUTO ? f->auto_variant : f->opt.variant;
+}
+
+static uint32_t pick_chunk(const fsm *f, uint64_t len_bytes, uint32_t T)
+{
+    if (f->opt.chunk_bytes) return f->opt.chunk_bytes;
+    // enough chunks to give every SM several resident tiles, chunks of 64 B .. 4 KiB
+    const uint64_t want_chunks = (uint64_t)f->num_sms * 2 * T;
+    uint64_t c = (len_bytes + want_chunks - 1) / want_chunks;
+    c = (c + 31) & ~31ull;
+    return (uint32_t)std::min<uint64_t>(4096, std::max<uint64_t>(64, c));
+}
+
+static int ensure_desc(fsm *f, size_t ntiles)
+{
+    if (ntiles <= f->desc_cap) return FSM_OK;
+    size_t cap = std::max<size_t>(ntiles, 1024);
+    cudaStreamSynchronize(f->stream);
+    cudaFree(f->d_desc);
+    f->d_desc = nullptr;
+    f->desc_cap = 0;
+    CK(cudaMalloc(&f->d_desc, cap * sizeof(TileDesc)));
+    CK(cudaMemset(f->d_desc, 0, cap * sizeof(TileDesc)));
+    f->desc_cap = cap;
+    return FSM_OK;
+}
+
+static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T);
+
+static int launch_run(fsm *f, const RunSpec &r)
+{
+    const int var = variant_of(f, r.force_variant);
+    const int K = kslots(r.k);
+    const uint32_t T = f->opt.threads_per_tile;
+    const bool bits = f->mode == FSM_INPUT_BITS_MSB;
+    const uint64_t len_bytes = bits ? r.len_sym / 8 : r.len_sym;
+    const uint32_t chunk = pick_chunk(f, len_bytes, T);
+    const uint64_t tile_bytes = (uint64_t)T * chunk;
+    uint64_t ntiles64 = (len_bytes + tile_bytes - 1) / tile_bytes;
+    if (ntiles64 == 0) ntiles64 = 1;
+    if (ntiles64 > 0x7FFFFFFFull) return FSM_EINVAL;
+    const uint32_t ntiles = (uint32_t)ntiles64;
+    int rc;
+
+    Params p{};
+    p.in = r.in;
+    p.len = len_bytes;
+    p.chunk = chunk;
+    p.ntiles = ntiles;
+    p.k = r.k;
+    p.aligned = ((uintptr_t)r.in & 31) == 0;
+    p.table = f->d_img[var];
+    p.n_states = f->dfa.n;
+    p.table_bytes = f->img_bytes[var];
+    p.lb = f->d_lb;
+    p.nimg = f->d_nimg;
+    p.keyed = r.keyed;
+    p.start_state = r.start_state;
+    p.start_dev = r.start_dev;
+    p.halo_byte = r.halo_byte;
+    p.tail_bits = bits ? (uint32_t)(r.len_sym & 7) : 0;
+    p.bittab = f->d_bittab;
+    p.result = r.result;
+    p.stats = f->d_stats;
+    p.ticket = f->d_ticket;
+
+    const size_t smem = Layout(T, K, p.table_bytes).total;
+
+    if (r.merge == FSM_MERGE_SEQUENTIAL) {
+        if (r.keyed) return FSM_EINVAL;
+        return launch_seq(f, p, var, K, T);
+    }
+
+    if ((rc = ensure_desc(f, ntiles))) return rc;
+    p.desc = f->d_desc;
+    KernelFn fn = get_kernel(var, K);
+    CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)T, smem));
+    if (occ < 1) return FSM_EINVAL;
+    if (f->opt.ctas_per_sm) occ = std::min<int>(occ, (int)f->opt.ctas_per_sm);
+    const uint32_t grid = (uint32_t)std::min<uint64_t>(ntiles, (uint64_t)occ * f->num_sms);
+    f->epoch = (f->epoch + 1) & 0x3FFFFFFFu;
+    if (f->epoch == 0) f->epoch = 1;
+    p.epoch = f->epoch;
+    p.ticket_base = f->ticket_base;
+    fn<<<grid, T, smem, f->stream>>>(p);
+    CK(cudaGetLastError());
+    f->ticket_base += ntiles + grid;  // every CTA takes one ticket past the end
+    f->last.chunks = (len_bytes + chunk - 1) / chunk;
+    f->last.tiles = ntiles;
+    f->last.chunk_bytes = chunk;
+    f->last.threads_per_tile = T;
+    f->last.variant = var;
+    f->last.k_slots = K;
+    return FSM_OK;
+}
+
+// Sequential-merge ablation (Fig. 4a): local kernel over all chunks, then one walking CTA.
+static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T)
+{
+    const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
+    if (nch * K > f->seq_cap) {
+        cudaStreamSynchronize(f->stream);
+        cudaFree(f->seq.S);
+        cudaFree(f->seq.E);
+        cudaFree(f->seq.C);
+        f->seq = SeqBuf{};
+        f->seq_cap = 0;
+        CK(cudaMalloc(&f->seq.S, nch * K * 2));
+        CK(cudaMalloc(&f->seq.E, nch * K * 4));
+        CK(cudaMalloc(&f->seq.C, nch * K * 4));
+        f->seq_cap = nch * K;
+    }
+    SeqLocalFn lf;
+    SeqWalkFn wf;
+    get_seq(var, K, lf, wf);
+    const size_t smem_l = (p.table_bytes + 15) & ~15u;
+    CK(cudaFuncSetAttribute((const void *)lf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(smem_l, 16)));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lf, (int)T, std::max<size_t>(smem_l, 16)));
+    const uint64_t blocks = std::min<uint64_t>((nch + T - 1) / T, (uint64_t)std::max(occ, 1) * f->num_sms);
+    lf<<<(uint32_t)blocks, T, std::max<size_t>(smem_l, 16), f->stream>>>(p, f->seq);
+    CK(cudaGetLastError());
+    const size_t smem_w = seq_walk_smem(T, K, p.table_bytes);
+    CK(cudaFuncSetAttribute((const void *)wf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_w));
+    wf<<<1, T, smem_w, f->stream>>>(p, f->seq);
+    CK(cudaGetLastError());
+    f->last.chunks = nch;
+    f->last.tiles = 0;
+    f->last.chunk_bytes = p.chunk;
+    f->last.threads_per_tile = T;
+    f->last.variant = var;
+    f->last.k_slots = K;
+    return FSM_OK;
+}
+
+static int check_run_args(const fsm *f, const uint8_t *input, uint64_t len, uint32_t k)
+{
+    if (!f) return FSM_EINVAL;
+    if (k < 1 || k > FSM_KMAX || k > f->n_user) return FSM_EINVAL;
+    if (len > 0 && !input) return FSM_EINVAL;
+    return FSM_OK;
+}
+
+// Read result + stats of the run just enqueued (one small D2H), fill f->last.
+static int finish_sync(fsm *f, const DevResult *dres)
+{
+    DevResult *hr = f->h_result;
+    DevStats *hs = reinterpret_cast<DevStats *>(hr + 1);
+    CK(cudaMemcpyAsync(hr, dres, sizeof(DevResult), cudaMemcpyDeviceToHost, f->stream));
+    CK(cudaMemcpyAsync(hs, f->d_stats, sizeof(DevStats), cudaMemcpyDeviceToHost, f->stream));
+    CK(cudaStreamSynchronize(f->stream));
+    f->last.reexec_chunks = hs->reexec_chunks - f->stats_before.reexec_chunks;
+    f->last.reexec_symbols = hs->reexec_bytes - f->stats_before.reexec_bytes;
+    f->last.boundary_misses = hs->boundary_misses - f->stats_before.boundary_misses;
+    f->stats_before = *hs;
+    return FSM_OK;
+}
+
+static bool is_sink(const fsm *f, uint32_t s) { return f->dfa.sink != 0xFFFFFFFFu && s == f->dfa.sink; }
+
+extern "C" int fsm_run_spec_k_async(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k, fsm_result *dev_result)
+{
+    int rc = check_run_args(f, input, len, k);
+    if (rc) return rc;
+    if (!dev_result) return FSM_EINVAL;
+    RunSpec r{input, len, k, false, 0, f->start, nullptr, f->d_result, -1, f->opt.merge};
+    if ((rc = launch_run(f, r))) return rc;
+    CK(cudaMemcpyAsync(dev_result, f->d_result, sizeof(fsm_result), cudaMemcpyDeviceToDevice, f->stream));
+    return FSM_OK;
+}
+
+extern "C" int fsm_run_spec_k(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k, uint32_t *final_state,
+                              uint64_t *accept_count)
+{
+    int rc = check_run_args(f, input, len, k);
+    if (rc) return rc;
+    if (!final_state || !accept_count) return FSM_EINVAL;
+    RunSpec r{input, len, k, false, 0, f->start, nullptr, f->d_result, -1, f->opt.merge};
+    if ((rc = launch_run(f, r))) return rc;
+    if ((rc = finish_sync(f, f->d_result))) return rc;
+    if (is_sink(f, f->h_result->final_state)) return FSM_ESYMBOL;
+    *final_state = f->h_result->final_state;
+    *accept_count = f->h_result->count;
+    return FSM_OK;
+}
+
+// End-to-end over a host buffer: pieces copied H2D on a copy stream into two staging buffers,
+// each piece's kernel chained to the previous piece's result on the device.
+extern "C" int fsm_run_spec_k_host(fsm_t *f, const uint8_t *host_input, uint64_t len, uint32_t k,
+                                   uint32_t *final_state, uint64_t *accept_count)
+{
+    int rc = check_run_args(f, host_input, len, k);
+    if (rc) return rc;
+    if (!final_state || !accept_count) return FSM_EINVAL;
+    const bool bits = f->mode == FSM_INPUT_BITS_MSB;
+    const uint64_t nbytes = bits ? (len + 7) / 8 : len;
+    const size_t piece = (size_t)1 << 28;  // 256 MiB
+    if (!f->d_stage[0]) {
+        CK(cudaMalloc(&f->d_stage[0], piece + 64));
+        CK(cudaMalloc(&f->d_stage[1], piece + 64));
+        for (int i = 0; i < 2; i++) {
+            CK(cudaEventCreateWithFlags(&f->ev_copied[i], cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&f->ev_used[i], cudaEventDisableTiming));
+        }
+        CK(cudaStreamCreateWithFlags(&f->copy_stream, cudaStreamNonBlocking));
+        f->stage_bytes = piece;
+    }
+    // the stage buffers may still be read by a previous call's kernels
+    for (int i = 0; i < 2; i++) CK(cudaEventRecord(f->ev_used[i], f->stream));
+    const uint64_t npieces = nbytes == 0 ? 1 : (nbytes + piece - 1) / piece;
+    uint64_t chunks = 0, tiles = 0;
+    for (uint64_t pi = 0; pi < npieces; pi++) {
+        const int sb = (int)(pi & 1);
+        const uint64_t off = pi * piece;
+        const uint64_t nb = std::min<uint64_t>(piece, nbytes - std::min(nbytes, off));
+        CK(cudaStreamWaitEvent(f->copy_stream, f->ev_used[sb], 0));
+        if (nb) CK(cudaMemcpyAsync(f->d_stage[sb], host_input + off, nb, cudaMemcpyHostToDevice, f->copy_stream));
+        CK(cudaEventRecord(f->ev_copied[sb], f->copy_stream));
+        CK(cudaStreamWaitEvent(f->stream, f->ev_copied[sb], 0));
+        uint64_t sym = bits ? std::min<uint64_t>(len - off * 8, (uint64_t)nb * 8) : nb;
+        // chain: piece pi starts from piece pi-1's result (d_result[0]); it writes to d_result[pi&1 ^ ...]
+        DevResult *res = f->d_result + ((pi + 1) & 1);
+        const DevResult *prev = pi == 0 ? nullptr : f->d_result + (pi & 1);
+        RunSpec r{f->d_stage[sb], sym, k, false, 0, f->start, prev, res, -1, FSM_MERGE_PARALLEL};
+        if ((rc = launch_run(f, r))) return rc;
+        CK(cudaEventRecord(f->ev_used[sb], f->stream));
+        chunks += f->last.chunks;
+        tiles += f->last.tiles;
+    }
+    const DevResult *fin = f->d_result + (npieces & 1);
+    if ((rc = finish_sync(f, fin))) return rc;
+    f->last.chunks = chunks;
+    f->last.tiles = tiles;
+    if (is_sink(f, f->h_result->final_state)) return FSM_ESYMBOL;
+    *final_state = f->h_result->final_state;
+    *accept_count = f->h_result->count;
+    return FSM_OK;
+}
+
+// ------------------------------------------------------------------------------- shards ----
+extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const uint8_t *halo, uint32_t halo_len,
+                             uint32_t k, fsm_shard_map *out, fsm_shard_t **state)
+{
+    int rc = check_run_args(f, input, len, k);
+    if (rc) return rc;
+    if (!out || (halo_len > 0 && !halo)) return FSM_EINVAL;
+    uint32_t hb = 0;
+    const bool keyed = halo_len > 0;
+    if (keyed) {
+        uint8_t h = 0;
+        CK(cudaMemcpyAsync(&h, halo + halo_len - 1, 1, cudaMemcpyDeviceToHost, f->stream));
+        CK(cudaStreamSynchronize(f->stream));
+        hb = h;
+    }
+    RunSpec r{input, len, k, keyed, hb, f->start, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL};
+    if ((rc = launch_run(f, r))) return rc;
+    if ((rc = finish_sync(f, f->d_result))) return rc;
+    const DevResult *hr = f->h_result;
+    fsm_shard_map m{};
+    m.k = k;
+    if (!keyed) {
+        m.valid_mask = 1;
+        m.start[0] = f->start;
+        m.end[0] = hr->final_state;
+        m.count[0] = hr->count;
+    } else {
+        m.valid_mask = hr->valid_mask & ((1u << KMAX) - 1);
+        for (int s = 0; s < KMAX; s++) {
+            m.start[s] = hr->start[s];
+            m.end[s] = hr->end[s];
+            m.count[s] = hr->mcount[s];
+        }
+    }
+    *out = m;
+    if (state) {
+        fsm_shard *st = new (std::nothrow) fsm_shard();
+        if (!st) return FSM_ENOMEM;
+        st->input = input;
+        st->len = len;
+        st->k = k;
+        st->map = m;
+        *state = st;
+    }
+    return FSM_OK;
+}
+
+extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, uint32_t *end, uint64_t *count)
+{
+    if (!f || !st || !end || !count || true_start >= f->dfa.n) return FSM_EINVAL;
+    for (int s = 0; s < KMAX; s++)
+        if (((st->map.valid_mask >> s) & 1u) && st->map.start[s] == true_start) {
+            *end = st->map.end[s];
+            *count = st->map.count[s];
+            return FSM_OK;
+        }
+    const bool bits = f->mode == FSM_INPUT_BITS_MSB;
+    const uint64_t whole = bits ? st->len / 8 : st->len;
+    const int var = variant_of(f, -1);
+    FixParams fp{};
+    fp.in = st->input;
+    fp.len = whole;
+    fp.limit = (uint64_t)1 << 20;
+    fp.table = f->d_img[var];
+    fp.n_states = f->dfa.n;
+    fp.x = true_start;
+    fp.k = st->map.k;
+    fp.valid_mask = st->map.valid_mask;
+    for (int s = 0; s < KMAX; s++) {
+        fp.start[s] = st->map.start[s];
+        fp.end[s] = st->map.end[s];
+        fp.count[s] = st->map.count[s];
+    }
+    fp.out = f->d_fix;
+    FixFn fn = get_fix(var);
+    const size_t smem = std::max<uint32_t>(16, f->img_bytes[var]);
+    CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    fn<<<1, kThreads, smem, f->stream>>>(fp);
+    CK(cudaGetLastError());
+    unsigned long long h[4];
+    CK(cudaMemcpyAsync(h, f->d_fix, sizeof(h), cudaMemcpyDeviceToHost, f->stream));
+    CK(cudaStreamSynchronize(f->stream));
+    if (h[0]) {
+        *end = (uint32_t)h[1];
+        *count = h[2];
+        return FSM_OK;
+    }
+    // no convergence: exact parallel re-run of the shard from the true start
+    RunSpec r{st->input, st->len, st->k, false, 0, true_start, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL};
+    int rc = launch_run(f, r);
+    if (rc) return rc;
+    if ((rc = finish_sync(f, f->d_result))) return rc;
+    *end = f->h_result->final_state;
+    *count = f->h_result->count;
+    return FSM_OK;
+}
+
+extern "C" void fsm_shard_free(fsm_shard_t *st) { delete st; }
+
+extern "C" int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, fsm_shard_map *out)
+{
+    if (!a || !b || !out) return FSM_EINVAL;
+    fsm_shard_map r = *a;
+    r.valid_mask = 0;
+    for (int s = 0; s < KMAX; s++) {
+        if (!((a->valid_mask >> s) & 1u)) continue;
+        for (int j = 0; j < KMAX; j++)
+            if (((b->valid_mask >> j) & 1u) && b->start[j] == a->end[s]) {
+                r.end[s] = b->end[j];
+                r.count[s] = a->count[s] + b->count[j];
+                r.valid_mask |= 1u << s;
+                break;
+            }
+    }
+    *out = r;
+    return FSM_OK;
+}

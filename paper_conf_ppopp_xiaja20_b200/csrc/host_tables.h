@@ -1,0 +1,116 @@
+// host_tables.h -- host preprocessing at fsm_create: validation, sink state,
+// bit-mode widening, the look-back table and the per-variant device table images.
+// Pure host code (no CUDA calls) so that it is usable without a GPU.
+#pragma once
+#include <algorithm>
+#include <cstdint>
+#include <cstring>
+#include <vector>
+
+#include "speck_types.h"
+
+namespace speck {
+
+// The DFA as the kernels see it: 256 byte columns, internal ids (sink appended when alphabet <
+// 256 in byte mode), entries next | count where count = accept increments along the step (byte
+// mode: F[next]; bit mode: F-visits over the 8 MSB-first bits of the byte).
+struct ByteDFA {
+    uint32_t n = 0;                 // internal states
+    uint32_t sink = 0xFFFFFFFFu;    // internal sink id or none
+    std::vector<uint32_t> next;     // [n][256]
+    std::vector<uint8_t> inc;       // [n][256] accept increments (0..8)
+    std::vector<uint32_t> bittab;   // bit mode: [n][2] next | acc << 16 (tail bits)
+};
+
+inline int build_byte_dfa(const uint32_t *table, uint32_t n_states, uint32_t alphabet,
+                          const uint8_t *accept, bool bit_mode, ByteDFA &d)
+{
+    auto acc = [&](uint32_t s) -> uint8_t { return (accept && s < n_states && accept[s]) ? 1 : 0; };
+    if (!bit_mode) {
+        const bool need_sink = alphabet < 256;
+        d.n = n_states + (need_sink ? 1 : 0);
+        d.sink = need_sink ? n_states : 0xFFFFFFFFu;
+        d.next.assign((size_t)d.n * 256, 0);
+        d.inc.assign((size_t)d.n * 256, 0);
+        for (uint32_t s = 0; s < d.n; s++)
+            for (uint32_t c = 0; c < 256; c++) {
+                uint32_t t = (s == d.sink || c >= alphabet) ? d.sink : table[(size_t)s * alphabet + c];
+                d.next[(size_t)s * 256 + c] = t;
+                d.inc[(size_t)s * 256 + c] = acc(t);
+            }
+    } else {
+        // widening: T8[s][byte] = delta over the 8 bits MSB-first, C8 = F-visits on the way
+        d.n = n_states;
+        d.next.assign((size_t)d.n * 256, 0);
+        d.inc.assign((size_t)d.n * 256, 0);
+        d.bittab.assign((size_t)d.n * 2, 0);
+        for (uint32_t s = 0; s < d.n; s++) {
+            for (uint32_t b = 0; b < 2; b++) {
+                uint32_t t = table[(size_t)s * 2 + b];
+                d.bittab[(size_t)s * 2 + b] = t | ((uint32_t)acc(t) << 16);
+            }
+            for (uint32_t c = 0; c < 256; c++) {
+                uint32_t q = s, k = 0;
+                for (int i = 7; i >= 0; i--) {
+                    q = table[(size_t)q * 2 + ((c >> i) & 1)];
+                    k += acc(q);
+                }
+                d.next[(size_t)s * 256 + c] = q;
+                d.inc[(size_t)s * 256 + c] = (uint8_t)k;
+            }
+        }
+    }
+    return 0;
+}
+
+// Look-back table (reading A5): image of each byte ranked by preimage count, ties -> smaller id.
+// The internal sink is not a source: it is only ever entered through an out-of-alphabet byte,
+// whose image is then exactly {sink}.
+inline void build_lookback(const ByteDFA &d, uint16_t *lb, uint8_t *nimg)
+{
+    std::vector<uint32_t> pre(d.n);
+    std::vector<uint32_t> ids;
+    for (uint32_t c = 0; c < 256; c++) {
+        std::fill(pre.begin(), pre.end(), 0u);
+        for (uint32_t s = 0; s < d.n; s++)
+            if (s != d.sink) pre[d.next[(size_t)s * 256 + c]]++;
+        ids.clear();
+        for (uint32_t q = 0; q < d.n; q++)
+            if (pre[q]) ids.push_back(q);
+        std::stable_sort(ids.begin(), ids.end(), [&](uint32_t a, uint32_t b) {
+            return pre[a] != pre[b] ? pre[a] > pre[b] : a < b;
+        });
+        uint32_t m = (uint32_t)std::min<size_t>(ids.size(), KMAX);
+        nimg[c] = (uint8_t)m;
+        for (uint32_t i = 0; i < KMAX; i++) lb[c * KMAX + i] = i < m ? (uint16_t)ids[i] : (uint16_t)0xFFFF;
+    }
+}
+
+// Variant images (layouts documented in speck_kernel.cuh / DESIGN.md).
+inline std::vector<uint8_t> image_packed(const ByteDFA &d, bool wide)
+{
+    const uint32_t bytes = wide ? 8 : 4;
+    std::vector<uint8_t> img(256 * bytes, 0);
+    for (uint32_t c = 0; c < 256; c++)
+        for (uint32_t s = 0; s < d.n; s++)
+            img[c * bytes + s] = (uint8_t)(d.next[(size_t)s * 256 + c] | (d.inc[(size_t)s * 256 + c] << 4));
+    return img;
+}
+
+inline std::vector<uint8_t> image_b(const ByteDFA &d)
+{
+    std::vector<uint8_t> img((size_t)d.n * 512);
+    uint16_t *p = reinterpret_cast<uint16_t *>(img.data());
+    for (size_t i = 0; i < (size_t)d.n * 256; i++) p[i] = (uint16_t)(d.next[i] | ((uint32_t)d.inc[i] << 8));
+    return img;
+}
+
+inline std::vector<uint8_t> image_g(const ByteDFA &d)
+{
+    std::vector<uint8_t> img((size_t)d.n * 1024);
+    uint32_t *p = reinterpret_cast<uint32_t *>(img.data());
+    for (size_t i = 0; i < (size_t)d.n * 256; i++) p[i] = d.next[i] | ((uint32_t)d.inc[i] << 16);
+    return img;
+}
+
+}  // namespace speck

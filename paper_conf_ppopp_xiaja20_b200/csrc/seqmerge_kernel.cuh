@@ -1,0 +1,166 @@
+// seqmerge_kernel.cuh -- the sequential-merge ablation (Fig. 4a).
+//
+// Same local phase as the parallel path (Alg. 3, same chunking and look-back), but every chunk
+// writes its k-slot mapping to global memory and ONE thread then walks the chunks in order with
+// the true state: a speculated match takes the chunk's ending state, otherwise the chunk is
+// re-executed from the true state (same exact early-exit re-execution as the parallel path, so
+// the two differ only in the merge).  The walking CTA prefetches the next batch of mappings into
+// shared memory so the walk is bound by shared-memory latency, not HBM latency.  This is the
+// merge the paper shows to be the scalability bottleneck.
+#pragma once
+#include "speck_kernel.cuh"
+
+namespace speck {
+
+struct SeqBuf {
+    uint16_t *S;   // [nchunks][K]
+    uint32_t *E;   // [nchunks][K]
+    uint32_t *C;   // [nchunks][K]
+};
+
+template <int K, int VAR>
+__global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb)
+{
+    using TB = typename TableFor<VAR>::type;
+    extern __shared__ __align__(16) uint8_t smem[];
+    TB tb;
+    tb.setup(smem, p.table, p.n_states);
+    __syncthreads();
+    const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
+    const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
+    for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nch; g += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t b = g * p.chunk, e = min(b + p.chunk, p.len);
+        uint32_t S[K];
+        if (g == 0) {
+#pragma unroll
+            for (int s = 0; s < K; s++) S[s] = s == 0 ? start_state : NOSTATE;
+        } else {
+            const uint32_t c = __ldg(p.in + b - 1);
+            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), p.k);
+#pragma unroll
+            for (int s = 0; s < K; s++) S[s] = (uint32_t)s < ni ? (uint32_t)__ldg(p.lb + c * KMAX + s) : NOSTATE;
+        }
+        uint32_t cur[K], acc[K];
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            cur[s] = tb.init(S[s] == NOSTATE ? 0u : S[s]);
+            acc[s] = 0;
+        }
+        if (e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc);
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            sb.S[g * K + s] = (uint16_t)(S[s] == NOSTATE ? 0xFFFFu : S[s]);
+            sb.E[g * K + s] = tb.state_of(cur[s]);
+            sb.C[g * K + s] = tb.count_of(acc[s]);
+        }
+    }
+}
+
+template <int K, int VAR>
+__global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
+{
+    using TB = typename TableFor<VAR>::type;
+    extern __shared__ __align__(16) uint8_t smem[];
+    TB tb;
+    tb.setup(smem, p.table, p.n_states);
+    const uint32_t T = blockDim.x;
+    const uint32_t tb_bytes = (p.table_bytes + 15) & ~15u;
+    // double-buffered batches of T mappings
+    uint16_t *bS = reinterpret_cast<uint16_t *>(smem + tb_bytes);            // [2][T][K]
+    uint32_t *bE = reinterpret_cast<uint32_t *>(smem + tb_bytes + 2 * T * K * 2 + 16);
+    uint32_t *bC = bE + 2 * T * K;
+    const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
+    const uint64_t nbatch = (nch + T - 1) / T;
+    auto load = [&](uint64_t batch, int buf) {
+        const uint64_t g0 = batch * T;
+        for (uint32_t i = threadIdx.x; i < T * K; i += T) {
+            const uint64_t g = g0 + i / K;
+            if (g < nch) {
+                bS[buf * T * K + i] = sb.S[g0 * K + i];
+                bE[buf * T * K + i] = sb.E[g0 * K + i];
+                bC[buf * T * K + i] = sb.C[g0 * K + i];
+            }
+        }
+    };
+    load(0, 0);
+    __syncthreads();
+    uint32_t x = p.start_dev ? p.start_dev->final_state : p.start_state;
+    unsigned long long total = p.start_dev ? p.start_dev->count : 0ull;
+    unsigned long long reexec = 0, rebytes = 0;
+    for (uint64_t batch = 0; batch < nbatch; batch++) {
+        const int buf = batch & 1;
+        if (threadIdx.x != 0) {
+            if (batch + 1 < nbatch) load(batch + 1, buf ^ 1);
+        } else {
+            const uint64_t g0 = batch * T;
+            const uint32_t n = (uint32_t)((nch - g0) < T ? (nch - g0) : T);
+            for (uint32_t i = 0; i < n; i++) {
+                const uint16_t *Sg = bS + buf * T * K + i * K;
+                int hit = -1;
+#pragma unroll
+                for (int l = 0; l < K; l++)
+                    if (Sg[l] == x) hit = l;
+                if (hit >= 0) {
+                    total += bC[buf * T * K + i * K + hit];
+                    x = bE[buf * T * K + i * K + hit];
+                    continue;
+                }
+                // re-execute the chunk from the true state (Fig. 4a), early exit on convergence
+                const uint64_t b = (g0 + i) * p.chunk, e = min(b + p.chunk, p.len);
+                uint32_t y[K], cy[K];
+                bool pres[K];
+#pragma unroll
+                for (int l = 0; l < K; l++) {
+                    pres[l] = Sg[l] != 0xFFFFu;
+                    y[l] = pres[l] ? Sg[l] : 0u;
+                    cy[l] = 0;
+                }
+                uint32_t cx = 0, cyc = 0;
+                int conv = -1;
+                uint64_t pos = b;
+                while (conv < 0 && pos < e) {
+                    const typename TB::Row r = tb.row(__ldg(p.in + pos));
+                    x = tb.apply(r, x, cx);
+#pragma unroll
+                    for (int l = 0; l < K; l++) y[l] = tb.apply(r, y[l], cy[l]);
+#pragma unroll
+                    for (int l = 0; l < K; l++)
+                        if (pres[l] && conv < 0 && y[l] == x) {
+                            conv = l;
+                            cyc = cy[l];
+                        }
+                    pos++;
+                }
+                reexec++;
+                rebytes += pos - b;
+                if (conv >= 0) {
+                    total += (unsigned long long)cx - cyc + bC[buf * T * K + i * K + conv];
+                    x = bE[buf * T * K + i * K + conv];
+                } else {
+                    total += cx;
+                }
+            }
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        const uint32_t tail_byte = p.tail_bits ? __ldg(p.in + p.len) : 0u;
+        for (uint32_t i = 0; i < p.tail_bits; i++) {
+            const uint32_t en = __ldg(p.bittab + x * 2 + ((tail_byte >> (7 - i)) & 1u));
+            x = en & 0xFFFFu;
+            total += en >> 16;
+        }
+        p.result->final_state = x;
+        p.result->status = 0;
+        p.result->count = total;
+        atomicAdd(&p.stats->reexec_chunks, reexec);
+        atomicAdd(&p.stats->reexec_bytes, rebytes);
+    }
+}
+
+inline size_t seq_walk_smem(uint32_t T, int K, uint32_t table_bytes)
+{
+    return ((table_bytes + 15) & ~15u) + 2 * T * K * 2 + 16 + 2 * 2 * T * K * 4;
+}
+
+}  // namespace speck

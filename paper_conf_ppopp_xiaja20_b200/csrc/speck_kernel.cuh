@@ -1,0 +1,740 @@
+// speck_kernel.cuh -- the fused spec-k kernel for sm_100a (B200).
+//
+// One persistent CTA loop; each iteration takes the next tile from an atomic ticket (dynamic
+// tile ids => forward progress without co-residency assumptions) and runs the whole hot path:
+//
+//   a2  chunking: tile = blockDim.x chunks of p.chunk bytes, one chunk per thread;
+//       each thread streams its own chunk with 32-byte LDG.256 (full sectors) -- the paper's
+//       coalescing layout transformation realised on the fly, see DESIGN.md.
+//   a3  look-back speculation: S_j = top-k of image(x[b_j - 1]) (Alg. 3 l.3 P:207).
+//   a4  local processing: k independent lookup chains per chunk (Alg. 3) plus accept
+//       counts, k unrolled into registers.
+//   a5  warp merge: shuffle suffix scan of chunk mappings with the membership check of Alg. 1
+//       (P:121-143); an unmatched ending state marks the slot invalid (delayed re-execution,
+//       P:188-190) and records where it broke.
+//   a6  block merge: warp aggregates through shared memory, scanned by warp 0.
+//   a8  delayed, selective re-execution: only chunks whose (candidate) start was not speculated
+//       are re-executed, in lockstep with that chunk's speculated chains, stopping as soon as the
+//       re-executed run joins one of them (exact early exit).
+//   a7  grid merge: decoupled look-back over per-tile descriptors (replaces the paper's
+//       persistent-thread sequential global merge).
+//   a9  the last tile writes (final state, accept count) or the shard's k-slot mapping.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "speck_types.h"
+
+namespace speck {
+
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3 };
+constexpr int kThreads = 256;
+constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
+
+// ------------------------------------------------------------------------------- PTX helpers --
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(uint32_t *p, uint32_t v)
+{
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+struct Bytes32 {
+    uint32_t w[8];
+};
+// 256-bit non-coherent streaming load (SASS LDG.E.NA.ENL2.256): one full 32-byte sector per lane.
+__device__ __forceinline__ Bytes32 ldg256(const uint8_t *p)
+{
+    Bytes32 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.w[0]), "=r"(r.w[1]), "=r"(r.w[2]), "=r"(r.w[3]), "=r"(r.w[4]), "=r"(r.w[5]),
+                   "=r"(r.w[6]), "=r"(r.w[7])
+                 : "l"(p));
+    return r;
+}
+__device__ __forceinline__ uint4 ldg128(const uint8_t *p)
+{
+    return __ldg(reinterpret_cast<const uint4 *>(p));
+}
+
+// ------------------------------------------------------------------- table-placement variants --
+// Every variant exposes
+//   setup(smem, global image, n)       copy / expand the table into shared memory (once per CTA)
+//   init(s) / state_of(cur) / count_of(acc)
+//   step<K>(w, j, cur, acc)            advance all K chains by byte j of word w (the hot loop)
+//   row(c) / apply(row, st, cnt)       single-chain step used by re-execution
+// Entries carry the accept increment of the destination state (byte mode 0/1, bit mode 0..8).
+
+// P4/P8: the transition function of symbol c packed into one row of N <= 4 (8) byte fields,
+// field = next | count << 4.  The row address depends only on the input byte, so it is off the
+// dependency chain; one conflict-free LDS.32/LDS.64 serves all K chains, and each chain step is
+// a single PRMT (byte select by the current state).  Lane-replicated: lane l reads its own copy.
+template <int VAR>
+struct TablePacked {
+    static constexpr bool kWide = VAR == VAR_P8;
+    const uint8_t *sm;
+    uint32_t lanereg;
+    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t)
+    {
+        sm = s;
+        lanereg = (threadIdx.x & 31) * (kWide ? 8 : 4);
+        if (kWide) {
+            const uint2 *rows = static_cast<const uint2 *>(g);
+            for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
+                uint32_t c = i >> 5, l = i & 31;
+                reinterpret_cast<uint2 *>(s)[c * 32 + l] = __ldg(rows + c);
+            }
+        } else {
+            const uint32_t *rows = static_cast<const uint32_t *>(g);
+            for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
+                uint32_t c = i >> 5, l = i & 31;
+                reinterpret_cast<uint32_t *>(s)[c * 64 + l] = __ldg(rows + c);
+            }
+        }
+    }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur & 0xFu; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc) const { return acc >> 4; }
+
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    {
+        // address = c * 256 + lane * 4|8, built by one PRMT: byte1 <- byte j of w, byte0 <- lanereg
+        const uint32_t a = __byte_perm(w, lanereg, 0x5504u | (uint32_t(j) << 4));
+        if (kWide) {
+            const uint2 r = *reinterpret_cast<const uint2 *>(sm + a);
+#pragma unroll
+            for (int s = 0; s < K; s++) {
+                cur[s] = __byte_perm(r.x, r.y, cur[s]);
+                acc[s] += cur[s] & 0xF0u;
+            }
+        } else {
+            const uint32_t r = *reinterpret_cast<const uint32_t *>(sm + a);
+#pragma unroll
+            for (int s = 0; s < K; s++) {
+                cur[s] = __byte_perm(r, 0u, cur[s]);
+                acc[s] += cur[s] & 0xF0u;
+            }
+        }
+    }
+    using Row = uint2;
+    __device__ __forceinline__ Row row(uint32_t c) const
+    {
+        if (kWide) return *reinterpret_cast<const uint2 *>(sm + (c << 8) + lanereg);
+        return make_uint2(*reinterpret_cast<const uint32_t *>(sm + (c << 8) + lanereg), 0u);
+    }
+    __device__ __forceinline__ uint32_t apply(Row r, uint32_t st, uint32_t &cnt) const
+    {
+        const uint32_t f = __byte_perm(r.x, r.y, st) & 0xFFu;
+        cnt += f >> 4;
+        return f & 0xFu;
+    }
+};
+
+// B: u16 entries T[s][c] = next | count << 8 in shared memory (N <= 256; 512 B per state).
+struct TableB {
+    const uint8_t *sm;
+    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n)
+    {
+        sm = s;
+        const uint4 *src = static_cast<const uint4 *>(g);
+        uint4 *dst = reinterpret_cast<uint4 *>(s);
+        for (uint32_t i = threadIdx.x; i < n * 32; i += blockDim.x) dst[i] = __ldg(src + i);
+    }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc) const { return acc >> 8; }
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    {
+        const uint32_t c2 = j == 0 ? ((w << 1) & 0x1FEu) : ((w >> (8 * j - 1)) & 0x1FEu);
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            const uint32_t e = *reinterpret_cast<const uint16_t *>(sm + (cur[s] << 9) + c2);
+            const uint32_t nx = e & 0xFFu;
+            acc[s] += e - nx;
+            cur[s] = nx;
+        }
+    }
+    using Row = uint32_t;
+    __device__ __forceinline__ Row row(uint32_t c) const { return c << 1; }
+    __device__ __forceinline__ uint32_t apply(Row c2, uint32_t st, uint32_t &cnt) const
+    {
+        const uint32_t e = *reinterpret_cast<const uint16_t *>(sm + (st << 9) + c2);
+        cnt += e >> 8;
+        return e & 0xFFu;
+    }
+};
+
+// G: u32 entries T[s][c] = next | count << 16 in global memory (L2-resident), any N <= 65535.
+struct TableG {
+    const uint32_t *gt;
+    __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t) { gt = static_cast<const uint32_t *>(g); }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc) const { return acc; }
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    {
+        const uint32_t c = (w >> (8 * j)) & 0xFFu;
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            const uint32_t e = __ldg(gt + ((cur[s] << 8) | c));
+            acc[s] += e >> 16;
+            cur[s] = e & 0xFFFFu;
+        }
+    }
+    using Row = uint32_t;
+    __device__ __forceinline__ Row row(uint32_t c) const { return c; }
+    __device__ __forceinline__ uint32_t apply(Row c, uint32_t st, uint32_t &cnt) const
+    {
+        const uint32_t e = __ldg(gt + ((st << 8) | c));
+        cnt += e >> 16;
+        return e & 0xFFFFu;
+    }
+};
+
+template <int VAR> struct TableFor;
+template <> struct TableFor<VAR_P4> { using type = TablePacked<VAR_P4>; };
+template <> struct TableFor<VAR_P8> { using type = TablePacked<VAR_P8>; };
+template <> struct TableFor<VAR_B> { using type = TableB; };
+template <> struct TableFor<VAR_G> { using type = TableG; };
+
+// --------------------------------------------------------------------- a4: local processing --
+template <int K, class TB>
+__device__ __forceinline__ void process32(const TB &tb, const Bytes32 &x, uint32_t (&cur)[K], uint32_t (&acc)[K])
+{
+    if constexpr (K <= 4) {
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+#pragma unroll
+            for (int j = 0; j < 4; j++) tb.template step<K>(x.w[q], j, cur, acc);
+    } else {
+        uint32_t w[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++) w[q] = x.w[q];
+#pragma unroll 1
+        for (int q = 0; q < 8; q++) {
+#pragma unroll
+            for (int j = 0; j < 4; j++) tb.template step<K>(w[0], j, cur, acc);
+#pragma unroll
+            for (int r = 0; r < 7; r++) w[r] = w[r + 1];
+        }
+    }
+}
+
+// Alg. 3 over bytes [b, e) of the input: 32-byte blocks with two blocks in flight,
+// then the ragged tail byte by byte.
+template <int K, class TB>
+__device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restrict__ in, uint64_t b, uint64_t e,
+                                            bool aligned, uint32_t (&cur)[K], uint32_t (&acc)[K])
+{
+    const uint8_t *p = in + b;
+    const uint64_t n = e - b;
+    const uint64_t nblk = aligned ? (n >> 5) : 0;
+    if (nblk) {
+        Bytes32 x0 = ldg256(p), x1 = x0;
+        if (nblk > 1) x1 = ldg256(p + 32);
+        for (uint64_t i = 0; i < nblk; i++) {
+            Bytes32 x2 = x1;
+            if (i + 2 < nblk) x2 = ldg256(p + 32 * (i + 2));
+            process32<K>(tb, x0, cur, acc);
+            x0 = x1;
+            x1 = x2;
+        }
+    }
+    for (uint64_t i = nblk << 5; i < n; i++) {
+        const uint32_t c = __ldg(p + i);
+        tb.template step<K>(c, 0, cur, acc);
+    }
+}
+
+// --------------------------------------------------------- a5/a6: composition of mappings --
+// (L x R)[s]: a complete slot of L whose end state is a speculated start of R continues with R's
+// slot (which may itself be broken further on) and adds counts -- the membership check of
+// Alg. 1, all K compares unrolled into predicated selects (k is a compile-time
+// constant).  No match: the slot breaks at R's first chunk.
+template <int K>
+__device__ __forceinline__ void compose(uint32_t (&eob)[K], uint32_t (&cnt)[K], const uint32_t (&Sr)[K],
+                                        const uint32_t (&eobr)[K], const uint32_t (&cntr)[K], uint32_t first_r)
+{
+#pragma unroll
+    for (int s = 0; s < K; s++) {
+        const uint32_t x = eob[s];
+        if ((x >> 16) == COMPLETE) {
+            const uint32_t st = x & 0xFFFFu;
+            uint32_t ne = st | (first_r << 16), nc = 0;
+#pragma unroll
+            for (int j = 0; j < K; j++)
+                if (Sr[j] == st) {
+                    ne = eobr[j];
+                    nc = cntr[j];
+                }
+            eob[s] = ne;
+            cnt[s] += nc;
+        }
+    }
+}
+
+// Warp-level suffix scan (Kogge-Stone over shuffles): afterwards lane i holds the mapping of
+// elements [i, 32) keyed on its own start set.  first0 = chunk index of lane 0's element, step =
+// chunk distance between lanes.
+template <int K>
+__device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eob)[K], uint32_t (&cnt)[K], bool &ident,
+                                                 uint32_t first0, uint32_t step)
+{
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        uint32_t Sr[K], er[K], cr[K];
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            Sr[s] = __shfl_down_sync(0xFFFFFFFFu, S[s], d);
+            er[s] = __shfl_down_sync(0xFFFFFFFFu, eob[s], d);
+            cr[s] = __shfl_down_sync(0xFFFFFFFFu, cnt[s], d);
+        }
+        const bool ir = __shfl_down_sync(0xFFFFFFFFu, (int)ident, d) != 0;
+        if (lane + d < 32 && !ir && !ident) compose<K>(eob, cnt, Sr, er, cr, first0 + (lane + d) * step);
+    }
+}
+
+// ----------------------------------------------------------------- shared-memory layout ----
+struct Layout {
+    uint32_t qe, qc, sj, ws, we, wc, wi, total;
+    __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t table_bytes)
+    {
+        uint32_t o = (table_bytes + 15) & ~15u;
+        qe = o;  o += T * K * 4;
+        qc = o;  o += T * K * 4;
+        sj = o;  o += T * K * 2;
+        o = (o + 15) & ~15u;
+        ws = o;  o += 32 * K * 4;
+        we = o;  o += 32 * K * 4;
+        wc = o;  o += 32 * K * 4;
+        wi = o;  o += 32 * 4;
+        total = o;
+    }
+};
+
+// Per-tile context used by re-execution and the epilogue.
+struct TileCtx {
+    const uint8_t *in;
+    uint64_t len;
+    uint64_t tile_base;
+    uint32_t chunk;
+    uint32_t nch;       // non-empty chunks in this tile (>= 1)
+    bool aligned;
+    const uint32_t *Qe, *Qc;
+    const uint16_t *Sj;
+    DevStats *stats;
+};
+
+// a8: resolve a broken slot.  The run is in state `st` when entering chunk c of the tile, with
+// count n so far.  Re-execute chunk c from st in lockstep with the chunk's speculated chains
+// ("re-execute the next chunk with states[s]"); the moment the re-executed state equals a
+// speculated chain's state both runs coincide for the rest of the chunk, so the result is exact:
+// (that chain's path, n + cnt_x(p) - cnt_l(p) + its count).  Otherwise continue at chunk c+1.
+template <int K, class TB>
+__device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c, uint32_t n, uint32_t &out_st,
+                        uint32_t &out_n)
+{
+    for (;;) {
+        const uint64_t b = t.tile_base + (uint64_t)c * t.chunk;
+        const uint64_t e = min(b + t.chunk, t.len);
+        uint32_t y[K], cy[K];
+        bool pres[K];
+#pragma unroll
+        for (int l = 0; l < K; l++) {
+            const uint32_t sv = t.Sj[c * K + l];
+            pres[l] = sv != 0xFFFFu;
+            y[l] = pres[l] ? sv : 0u;
+            cy[l] = 0;
+        }
+        uint32_t cx = 0, cyc = 0;
+        int conv = -1;
+        uint64_t pos = b;
+        auto one = [&](uint32_t byte) {
+            const typename TB::Row r = tb.row(byte);
+            st = tb.apply(r, st, cx);
+#pragma unroll
+            for (int l = 0; l < K; l++) y[l] = tb.apply(r, y[l], cy[l]);
+#pragma unroll
+            for (int l = 0; l < K; l++)
+                if (pres[l] && conv < 0 && y[l] == st) {
+                    conv = l;
+                    cyc = cy[l];
+                }
+        };
+        if (t.aligned) {
+            while (conv < 0 && pos + 16 <= e) {
+                const uint4 v = ldg128(t.in + pos);
+                uint32_t used = 0;
+#pragma unroll 1
+                for (int q = 0; q < 16 && conv < 0; q++) {
+                    const uint32_t wq = q < 8 ? (q < 4 ? v.x : v.y) : (q < 12 ? v.z : v.w);
+                    one((wq >> (8 * (q & 3))) & 0xFFu);
+                    used++;
+                }
+                pos += used;
+            }
+        }
+        while (conv < 0 && pos < e) {
+            one(__ldg(t.in + pos));
+            pos++;
+        }
+        atomicAdd(&t.stats->reexec_chunks, 1ull);
+        atomicAdd(&t.stats->reexec_bytes, (unsigned long long)(pos - b));
+        uint32_t x;
+        if (conv >= 0) {
+            n += cx - cyc + t.Qc[c * K + conv];
+            x = t.Qe[c * K + conv];
+        } else {
+            n += cx;
+            if (c + 1 >= t.nch) {
+                out_st = st;
+                out_n = n;
+                return;
+            }
+            x = st | ((c + 1) << 16);
+#pragma unroll
+            for (int l = 0; l < K; l++)
+                if (t.Sj[(c + 1) * K + l] == st) {
+                    x = t.Qe[(c + 1) * K + l];
+                    n += t.Qc[(c + 1) * K + l];
+                }
+        }
+        if ((x >> 16) == COMPLETE) {
+            out_st = x & 0xFFFFu;
+            out_n = n;
+            return;
+        }
+        st = x & 0xFFFFu;
+        c = x >> 16;
+    }
+}
+
+// ------------------------------------------------------------------------------- the kernel --
+template <int K, int VAR>
+__global__ void __launch_bounds__(kThreads) speck_kernel(Params p)
+{
+    using TB = typename TableFor<VAR>::type;
+    extern __shared__ __align__(16) uint8_t smem[];
+    __shared__ uint32_t s_tile;
+
+    const uint32_t T = blockDim.x;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = T >> 5;
+    const uint32_t j = threadIdx.x;
+
+    TB tb;
+    tb.setup(smem, p.table, p.n_states);
+    const Layout L(T, K, p.table_bytes);
+    uint32_t *Qe = reinterpret_cast<uint32_t *>(smem + L.qe);
+    uint32_t *Qc = reinterpret_cast<uint32_t *>(smem + L.qc);
+    uint16_t *Sj = reinterpret_cast<uint16_t *>(smem + L.sj);
+    uint32_t *wS = reinterpret_cast<uint32_t *>(smem + L.ws);
+    uint32_t *wE = reinterpret_cast<uint32_t *>(smem + L.we);
+    uint32_t *wC = reinterpret_cast<uint32_t *>(smem + L.wc);
+    uint32_t *wI = reinterpret_cast<uint32_t *>(smem + L.wi);
+
+    const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
+    const unsigned long long start_count = p.start_dev ? p.start_dev->count : 0ull;
+    const uint32_t ksel = p.k;
+
+    for (;;) {
+        __syncthreads();  // smem reuse across tiles; also orders the table setup
+        if (threadIdx.x == 0) s_tile = atomicAdd(p.ticket, 1u) - p.ticket_base;
+        __syncthreads();
+        const uint32_t tile = s_tile;
+        if (tile >= p.ntiles) break;
+
+        const uint64_t tile_base = (uint64_t)tile * T * p.chunk;
+        const uint64_t b = tile_base + (uint64_t)j * p.chunk;
+        const bool first_chunk = tile == 0 && j == 0;
+        const bool empty = b >= p.len && !first_chunk;
+        const uint64_t e = b >= p.len ? b : min(b + p.chunk, p.len);
+
+        // ---- a3: speculated start set
+        uint32_t S[K];
+        if (first_chunk && !p.keyed) {
+#pragma unroll
+            for (int s = 0; s < K; s++) S[s] = s == 0 ? start_state : NOSTATE;
+        } else {
+            uint32_t c = 0;
+            if (first_chunk) c = p.halo_byte;
+            else if (!empty) c = __ldg(p.in + b - 1);
+            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
+#pragma unroll
+            for (int s = 0; s < K; s++) S[s] = (!empty && (uint32_t)s < ni) ? (uint32_t)__ldg(p.lb + c * KMAX + s) : NOSTATE;
+        }
+
+        // ---- a4: local processing
+        uint32_t cur[K], acc[K];
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            cur[s] = tb.init(S[s] == NOSTATE ? 0u : S[s]);
+            acc[s] = 0;
+        }
+        if (!empty && e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc);
+        uint32_t eob[K], cnt[K];
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            eob[s] = S[s] == NOSTATE ? (ABSENT << 16) : (tb.state_of(cur[s]) | (COMPLETE << 16));
+            cnt[s] = tb.count_of(acc[s]);
+        }
+        bool ident = empty;
+
+        // ---- a5: warp stage (chunks warp*32 .. warp*32+31)
+        warp_suffix_scan<K>(S, eob, cnt, ident, (uint32_t)warp * 32, 1);
+
+        // ---- a6: block stage
+        if (lane == 0) {
+#pragma unroll
+            for (int s = 0; s < K; s++) {
+                wS[warp * K + s] = S[s];
+                wE[warp * K + s] = eob[s];
+                wC[warp * K + s] = cnt[s];
+            }
+            wI[warp] = ident;
+        }
+        __syncthreads();
+        if (warp == 0) {
+            uint32_t S2[K], e2[K], c2[K];
+            bool id2 = true;
+            if (lane < W) {
+#pragma unroll
+                for (int s = 0; s < K; s++) {
+                    S2[s] = wS[lane * K + s];
+                    e2[s] = wE[lane * K + s];
+                    c2[s] = wC[lane * K + s];
+                }
+                id2 = wI[lane] != 0;
+            } else {
+#pragma unroll
+                for (int s = 0; s < K; s++) S2[s] = NOSTATE, e2[s] = ABSENT << 16, c2[s] = 0;
+            }
+            warp_suffix_scan<K>(S2, e2, c2, id2, 0, 32);
+            __syncwarp();
+            if (lane < W) {
+#pragma unroll
+                for (int s = 0; s < K; s++) {
+                    wE[lane * K + s] = e2[s];
+                    wC[lane * K + s] = c2[s];
+                }
+            }
+        }
+        __syncthreads();
+        if (warp + 1 < W && !ident && wI[warp + 1] == 0) {
+            uint32_t Sr[K], er[K], cr[K];
+#pragma unroll
+            for (int s = 0; s < K; s++) {
+                Sr[s] = wS[(warp + 1) * K + s];
+                er[s] = wE[(warp + 1) * K + s];
+                cr[s] = wC[(warp + 1) * K + s];
+            }
+            compose<K>(eob, cnt, Sr, er, cr, (uint32_t)(warp + 1) * 32);
+        }
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            Qe[j * K + s] = eob[s];
+            Qc[j * K + s] = cnt[s];
+            Sj[j * K + s] = (uint16_t)(S[s] == NOSTATE ? 0xFFFFu : S[s]);
+        }
+        __syncthreads();
+
+        if (warp != 0) continue;
+
+        // ================= warp 0: tile epilogue (pre-resolution, look-back, publication) =====
+        TileCtx t;
+        t.in = p.in;
+        t.len = p.len;
+        t.tile_base = tile_base;
+        t.chunk = p.chunk;
+        {
+            const uint64_t rem = p.len > tile_base ? p.len - tile_base : 0;
+            const uint64_t nch = (rem + p.chunk - 1) / p.chunk;
+            t.nch = (uint32_t)(nch < 1 ? 1 : (nch > T ? T : nch));
+        }
+        t.aligned = p.aligned != 0;
+        t.Qe = Qe;
+        t.Qc = Qc;
+        t.Sj = Sj;
+        t.stats = p.stats;
+
+        // a8 (tile candidates): resolve the broken slots of the tile aggregate Q_0 so that the
+        // published aggregate is complete on every speculated tile start.
+        if (lane < K) {
+            const uint32_t x = Qe[lane];
+            if ((x >> 16) < ABSENT) {
+                uint32_t st, n;
+                resolve<K>(tb, t, x & 0xFFFFu, x >> 16, Qc[lane], st, n);
+                Qe[lane] = st | (COMPLETE << 16);
+                Qc[lane] = n;
+            }
+        }
+        __syncwarp();
+
+        // a7: publish the aggregate A_b
+        TileDesc *D = p.desc + tile;
+        if (lane < K) {
+            const uint32_t sv = Sj[lane];
+            D->astart[lane] = sv == 0xFFFFu ? NOSTATE : sv;
+            D->aend[lane] = Qe[lane] & 0xFFFFu;
+            D->acnt[lane] = Qc[lane];
+        }
+        __threadfence();
+        __syncwarp();
+        const uint32_t ep = p.epoch << 2;
+        if (lane == 0) st_release(&D->flag, ep | ST_A);
+
+        // a7: decoupled look-back -> exclusive prefix E (lane s = shard slot s)
+        uint32_t Es = 0;
+        unsigned long long Ec = 0;
+        bool Ev = false;
+        int64_t m;
+        {
+            int64_t base = (int64_t)tile - 1;
+            for (;;) {
+                const int64_t tt = base - lane;
+                uint32_t st = ST_P;
+                if (tt >= 0) {
+                    const uint32_t f = ld_acquire(&p.desc[tt].flag);
+                    st = (f & ~3u) == ep ? (f & 3u) : (uint32_t)ST_X;
+                }
+                const unsigned pm = __ballot_sync(0xFFFFFFFFu, st == ST_P);
+                const unsigned xm = __ballot_sync(0xFFFFFFFFu, st == ST_X);
+                const int fp = pm ? __ffs(pm) - 1 : 32;
+                const unsigned before = fp >= 32 ? 0xFFFFFFFFu : ((1u << fp) - 1u);
+                if (xm & before) {
+                    __nanosleep(100);
+                    continue;
+                }
+                if (fp < 32) {
+                    m = base - fp;
+                    break;
+                }
+                base -= 32;
+            }
+        }
+        auto load_P = [&](int64_t tt) {
+            const TileDesc *Dt = p.desc + tt;
+            while (ld_acquire(&Dt->flag) != (ep | ST_P)) __nanosleep(64);
+            const uint32_t pmask = __ldcg(&Dt->pmask);
+            Ev = lane < KMAX && ((pmask >> lane) & 1u);
+            if (lane < KMAX) {
+                Es = __ldcg(&Dt->pstate[lane]);
+                Ec = __ldcg(&Dt->pcnt[lane]);
+            }
+        };
+        if (m < 0) {
+            if (!p.keyed) {
+                Ev = lane == 0;
+                Es = start_state;
+                Ec = start_count;
+            } else {
+                const uint32_t c = p.halo_byte;
+                const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
+                Ev = (uint32_t)lane < ni;
+                Es = Ev ? (uint32_t)__ldg(p.lb + c * KMAX + lane) : 0u;
+                Ec = 0;
+            }
+        } else {
+            load_P(m);
+        }
+        for (int64_t tt = m + 1; tt < (int64_t)tile; tt++) {
+            const TileDesc *Dt = p.desc + tt;
+            const uint32_t f0 = __shfl_sync(0xFFFFFFFFu, ld_acquire(&Dt->flag), 0);
+            if ((f0 & 3u) == ST_P) {
+                load_P(tt);
+                continue;
+            }
+            // each lane acquires for itself before reading the A payload
+            while ((ld_acquire(&Dt->flag) & ~3u) != ep) __nanosleep(32);
+            bool hit = false;
+            if (Ev) {
+#pragma unroll 4
+                for (int l = 0; l < K; l++) {
+                    if (__ldcg(&Dt->astart[l]) == Es) {
+                        const uint32_t ne = __ldcg(&Dt->aend[l]);
+                        Ec += __ldcg(&Dt->acnt[l]);
+                        Es = ne;
+                        hit = true;
+                        break;
+                    }
+                }
+            }
+            if (__ballot_sync(0xFFFFFFFFu, Ev && !hit)) load_P(tt);  // a tile-boundary miss upstream
+        }
+
+        // own inclusive prefix P_b = E then A_b; a tile-boundary miss resolves through chunk 0.
+        uint32_t Ps = 0;
+        unsigned long long Pc = 0;
+        if (Ev) {
+            bool hit = false;
+#pragma unroll
+            for (int l = 0; l < K; l++)
+                if (!hit && Sj[l] == Es) {
+                    Ps = Qe[l] & 0xFFFFu;
+                    Pc = Ec + Qc[l];
+                    hit = true;
+                }
+            if (!hit) {
+                uint32_t st, n;
+                resolve<K>(tb, t, Es, 0, 0, st, n);
+                Ps = st;
+                Pc = Ec + n;
+                atomicAdd(&p.stats->boundary_misses, 1ull);
+            }
+        }
+        const unsigned vmask = __ballot_sync(0xFFFFFFFFu, Ev);
+        if (lane < KMAX) {
+            D->pstate[lane] = Ps;
+            D->pcnt[lane] = Pc;
+        }
+        if (lane == 0) D->pmask = vmask;
+        __threadfence();
+        __syncwarp();
+        if (lane == 0) st_release(&D->flag, ep | ST_P);
+
+        // a9: the last tile writes the result (bit-mode tail applied here)
+        if (tile == p.ntiles - 1) {
+            uint32_t x = Ps;
+            unsigned long long cc = Pc;
+            if (Ev && p.tail_bits) {
+                const uint32_t tail_byte = __ldg(p.in + p.len);
+                for (uint32_t i = 0; i < p.tail_bits; i++) {
+                    const uint32_t bit = (tail_byte >> (7 - i)) & 1u;
+                    const uint32_t en = __ldg(p.bittab + x * 2 + bit);
+                    x = en & 0xFFFFu;
+                    cc += en >> 16;
+                }
+            }
+            DevResult *R = p.result;
+            if (!p.keyed) {
+                if (lane == 0) {
+                    R->final_state = x;
+                    R->status = 0;
+                    R->count = cc;
+                }
+            } else {
+                const uint32_t c = p.halo_byte;
+                const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
+                if (lane < KMAX) {
+                    R->start[lane] = (uint32_t)lane < ni ? (uint32_t)__ldg(p.lb + c * KMAX + lane) : NOSTATE;
+                    R->end[lane] = x;
+                    R->mcount[lane] = cc;
+                }
+                if (lane == 0) {
+                    R->valid_mask = vmask;
+                    R->k = ksel;
+                    R->status = 0;
+                }
+            }
+        }
+    }
+}
+
+}  // namespace speck

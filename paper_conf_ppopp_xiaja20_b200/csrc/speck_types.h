@@ -1,0 +1,83 @@
+// speck_types.h -- structures shared by the host side (fsmspec.cu) and the kernels (speck_kernel.cuh).
+#pragma once
+#include <cstdint>
+
+namespace speck {
+
+constexpr int KMAX = 16;
+
+// ---- slot encoding inside a mapping (the merge element) ---------------------------------------
+// eob = state | brk << 16:  brk == COMPLETE : the run of this slot reaches the end of the range
+//                           brk == ABSENT   : the slot holds no speculated state (|image| < k)
+//                           otherwise       : the run breaks (no speculated match) when entering
+//                                             chunk `brk` of the tile in state `state` -- the
+//                                             paper's "invalid" slot plus where it broke.
+constexpr uint32_t COMPLETE = 0xFFFFu;
+constexpr uint32_t ABSENT = 0xFFFEu;
+constexpr uint32_t NOSTATE = 0xFFFFu;  // start-set sentinel: never equal to a state id
+
+enum Status : uint32_t { ST_X = 0, ST_A = 1, ST_P = 2 };
+
+// One descriptor per tile for the decoupled look-back.  The flag carries the
+// run epoch so descriptors never need clearing between runs.  A payload: the tile's aggregate
+// mapping keyed on its first chunk's start set.  P payload: the inclusive prefix -- a mapping
+// keyed on the shard's start set (one slot in known-start mode).
+struct __align__(128) TileDesc {
+    uint32_t flag;                 // epoch << 2 | Status
+    uint32_t pmask;                // P: valid slots
+    uint32_t astart[KMAX];         // A: start set of the tile's first chunk (NOSTATE = absent)
+    uint32_t aend[KMAX];           // A: end state per slot (ABSENT slots: unspecified)
+    uint32_t acnt[KMAX];           // A: accept count per slot within the tile
+    uint32_t pstate[KMAX];         // P: state after this tile, per shard slot
+    unsigned long long pcnt[KMAX]; // P: count up to and including this tile, per shard slot
+};
+
+struct DevStats {
+    unsigned long long reexec_chunks;
+    unsigned long long reexec_bytes;
+    unsigned long long boundary_misses;
+    unsigned long long pad;
+};
+
+// Result area written by the last tile.
+struct DevResult {
+    uint32_t final_state;   // known-start mode
+    uint32_t status;
+    unsigned long long count;
+    // keyed mode: the shard map
+    uint32_t valid_mask;
+    uint32_t k;
+    uint32_t start[KMAX];
+    uint32_t end[KMAX];
+    unsigned long long mcount[KMAX];
+};
+
+struct Params {
+    const uint8_t *in;             // input bytes of this run (bit mode: packed bytes)
+    uint64_t len;                  // whole bytes processed by the tiles
+    uint32_t chunk;                // bytes per chunk (multiple of 32)
+    uint32_t ntiles;
+    uint32_t k;                    // speculated states in use (<= template K)
+    uint32_t aligned;              // `in` is 32-byte aligned
+    const void *table;             // variant image in global memory
+    uint32_t n_states;             // internal states (incl. sink)
+    uint32_t table_bytes;          // bytes of the shared-memory table image (0 for G)
+    const uint16_t *lb;            // look-back table [256][KMAX]
+    const uint8_t *nimg;           // min(|image(c)|, KMAX)
+    TileDesc *desc;
+    uint32_t *ticket;
+    uint32_t ticket_base;
+    uint32_t epoch;
+    // start of the run
+    uint32_t keyed;                // 0: known start; 1: keyed on S_g = LB[halo]
+    uint32_t start_state;          // known start (ignored if start_dev)
+    const DevResult *start_dev;    // optional: known start (final_state, count) from a previous piece
+    uint32_t halo_byte;            // keyed mode
+    // bit-mode tail (applied by the last tile)
+    uint32_t tail_bits;            // the byte holding them is in[len]
+    const uint32_t *bittab;        // [n_states][2]: next | acc << 16
+    DevResult *result;
+    DevStats *stats;
+};
+
+}  // namespace speck

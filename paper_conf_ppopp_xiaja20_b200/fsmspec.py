@@ -1,0 +1,236 @@
+"""Thin ctypes binding of libfsmspec (include/fsmspec.h) -- argument marshalling only.
+
+Every step of the spec-k path runs in the CUDA kernels behind the C ABI; there is no CPU
+fallback: if libfsmspec.so is missing this module raises on import.  Torch is used only to
+hand over device pointers and streams (``tensor.data_ptr()``, ``stream.cuda_stream``).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+SO_PATH = os.path.join(_HERE, "libfsmspec.so")
+
+FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5
+FSM_INPUT_BYTES, FSM_INPUT_BITS_MSB = 0, 1
+FSM_KMAX = 16
+FSM_VARIANT_AUTO, FSM_VARIANT_P4, FSM_VARIANT_P8, FSM_VARIANT_B, FSM_VARIANT_G = -1, 0, 1, 2, 3
+VARIANT_NAMES = {0: "P4", 1: "P8", 2: "B", 3: "G"}
+FSM_MERGE_PARALLEL, FSM_MERGE_SEQUENTIAL = 0, 1
+
+# every symbol declared in include/fsmspec.h
+EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_set_stream",
+           "fsm_run_spec_k", "fsm_run_spec_k_async", "fsm_run_spec_k_host", "fsm_set_options",
+           "fsm_get_options", "fsm_get_stats", "fsm_run_shard", "fsm_shard_fixup", "fsm_shard_free",
+           "fsm_map_compose", "fsm_lookback_table", "fsm_version")
+
+
+class fsm_options(ctypes.Structure):
+    _fields_ = [("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
+                ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32)]
+
+
+class fsm_stats(ctypes.Structure):
+    _fields_ = [("chunks", ctypes.c_uint64), ("tiles", ctypes.c_uint64), ("reexec_chunks", ctypes.c_uint64),
+                ("reexec_symbols", ctypes.c_uint64), ("boundary_misses", ctypes.c_uint64),
+                ("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
+                ("variant", ctypes.c_uint32), ("k_slots", ctypes.c_uint32)]
+
+
+class fsm_shard_map(ctypes.Structure):
+    _fields_ = [("k", ctypes.c_uint32), ("valid_mask", ctypes.c_uint32),
+                ("start", ctypes.c_uint32 * FSM_KMAX), ("end", ctypes.c_uint32 * FSM_KMAX),
+                ("count", ctypes.c_uint64 * FSM_KMAX)]
+
+    def slots(self):
+        return [(int(self.start[s]), int(self.end[s]), int(self.count[s]))
+                for s in range(FSM_KMAX) if (self.valid_mask >> s) & 1]
+
+
+class FsmError(RuntimeError):
+    def __init__(self, status: int, what: str = ""):
+        self.status = status
+        super().__init__(f"{what}: {lib().fsm_strerror(status).decode()} ({status})")
+
+
+class SymbolError(FsmError):
+    pass
+
+
+_lib = None
+_P = ctypes.c_void_p
+_U32, _U64, _I32 = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int32
+
+
+def lib() -> ctypes.CDLL:
+    """Load libfsmspec.so.  Raises if it has not been built -- there is no fallback path."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(SO_PATH):
+            raise ImportError(f"{SO_PATH} is not built; run `python -c 'import __graft_entry__ as g; g.build()'`")
+        l = ctypes.CDLL(SO_PATH)
+        sig = {
+            "fsm_create": (_I32, [_P, _U32, _U32, _U32, _P, ctypes.POINTER(_P)]),
+            "fsm_create_ex": (_I32, [_P, _U32, _U32, _U32, _P, _U32, ctypes.POINTER(_P)]),
+            "fsm_destroy": (None, [_P]),
+            "fsm_strerror": (ctypes.c_char_p, [_I32]),
+            "fsm_set_stream": (_I32, [_P, _P]),
+            "fsm_run_spec_k": (_I32, [_P, _P, _U64, _U32, ctypes.POINTER(_U32), ctypes.POINTER(_U64)]),
+            "fsm_run_spec_k_async": (_I32, [_P, _P, _U64, _U32, _P]),
+            "fsm_run_spec_k_host": (_I32, [_P, _P, _U64, _U32, ctypes.POINTER(_U32), ctypes.POINTER(_U64)]),
+            "fsm_set_options": (_I32, [_P, ctypes.POINTER(fsm_options)]),
+            "fsm_get_options": (_I32, [_P, ctypes.POINTER(fsm_options)]),
+            "fsm_get_stats": (_I32, [_P, ctypes.POINTER(fsm_stats)]),
+            "fsm_run_shard": (_I32, [_P, _P, _U64, _P, _U32, _U32, ctypes.POINTER(fsm_shard_map),
+                                     ctypes.POINTER(_P)]),
+            "fsm_shard_fixup": (_I32, [_P, _P, _U32, ctypes.POINTER(_U32), ctypes.POINTER(_U64)]),
+            "fsm_shard_free": (None, [_P]),
+            "fsm_map_compose": (_I32, [ctypes.POINTER(fsm_shard_map), ctypes.POINTER(fsm_shard_map),
+                                       ctypes.POINTER(fsm_shard_map)]),
+            "fsm_lookback_table": (_I32, [_P, _U32, _U32, _U32, _P, _P]),
+            "fsm_version": (ctypes.c_char_p, []),
+        }
+        for name, (res, args) in sig.items():
+            fn = getattr(l, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = l
+    return _lib
+
+
+def _check(rc: int, what: str) -> None:
+    if rc == FSM_ESYMBOL:
+        raise SymbolError(rc, what)
+    if rc != FSM_OK:
+        raise FsmError(rc, what)
+
+
+def _ptr(x) -> int:
+    """Device or host address of a torch tensor / numpy array / int."""
+    if x is None:
+        return 0
+    if isinstance(x, int):
+        return x
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    return int(x.data_ptr())
+
+
+def lookback_table(table: np.ndarray, bit_mode: bool = False):
+    """fsm_lookback_table (host only): (lb [256, 16] uint16, nimg [256] uint8)."""
+    t = np.ascontiguousarray(table, dtype=np.uint32)
+    lb = np.zeros((256, FSM_KMAX), np.uint16)
+    ni = np.zeros(256, np.uint8)
+    _check(lib().fsm_lookback_table(t.ctypes.data, t.shape[0], t.shape[1],
+                                    FSM_INPUT_BITS_MSB if bit_mode else FSM_INPUT_BYTES,
+                                    lb.ctypes.data, ni.ctypes.data), "fsm_lookback_table")
+    return lb, ni
+
+
+def map_compose(a: fsm_shard_map, b: fsm_shard_map) -> fsm_shard_map:
+    out = fsm_shard_map()
+    _check(lib().fsm_map_compose(ctypes.byref(a), ctypes.byref(b), ctypes.byref(out)), "fsm_map_compose")
+    return out
+
+
+class FSM:
+    """One handle = one DFA on the current CUDA device (fsm_create_ex)."""
+
+    def __init__(self, table, start: int, accept=None, bit_mode: bool = False):
+        t = np.ascontiguousarray(table, dtype=np.uint32)
+        self.n_states, self.alphabet = int(t.shape[0]), int(t.shape[1])
+        self.bit_mode = bit_mode
+        acc = None if accept is None else np.ascontiguousarray(accept, dtype=np.uint8)
+        h = _P()
+        _check(lib().fsm_create_ex(t.ctypes.data, self.n_states, self.alphabet, start,
+                                   acc.ctypes.data if acc is not None else None,
+                                   FSM_INPUT_BITS_MSB if bit_mode else FSM_INPUT_BYTES, ctypes.byref(h)),
+               "fsm_create")
+        self._h = h
+
+    @classmethod
+    def from_dfa(cls, dfa) -> "FSM":
+        return cls(dfa.table, dfa.start, dfa.accept, dfa.bit_mode)
+
+    def close(self) -> None:
+        if getattr(self, "_h", None):
+            lib().fsm_destroy(self._h)
+            self._h = None
+
+    __del__ = close
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # ---------------------------------------------------------------------------- configuration
+    def set_stream(self, stream) -> None:
+        s = 0 if stream is None else (stream if isinstance(stream, int) else stream.cuda_stream)
+        _check(lib().fsm_set_stream(self._h, s), "fsm_set_stream")
+
+    def set_options(self, chunk_bytes: int = 0, threads_per_tile: int = 0, variant: int = FSM_VARIANT_AUTO,
+                    merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0) -> None:
+        o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm)
+        _check(lib().fsm_set_options(self._h, ctypes.byref(o)), "fsm_set_options")
+
+    def options(self) -> dict:
+        o = fsm_options()
+        _check(lib().fsm_get_options(self._h, ctypes.byref(o)), "fsm_get_options")
+        return {n: getattr(o, n) for n, _ in o._fields_}
+
+    def stats(self) -> dict:
+        s = fsm_stats()
+        _check(lib().fsm_get_stats(self._h, ctypes.byref(s)), "fsm_get_stats")
+        return {n: int(getattr(s, n)) for n, _ in s._fields_}
+
+    # ---------------------------------------------------------------------------------- runs
+    def run_spec_k(self, inp, length: int, k: int) -> tuple[int, int]:
+        """fsm_run_spec_k over a device-resident input (torch CUDA tensor or device address)."""
+        q, n = _U32(), _U64()
+        _check(lib().fsm_run_spec_k(self._h, _ptr(inp), length, k, ctypes.byref(q), ctypes.byref(n)),
+               "fsm_run_spec_k")
+        return int(q.value), int(n.value)
+
+    def run_spec_k_async(self, inp, length: int, k: int, dev_result) -> None:
+        """fsm_run_spec_k_async: enqueue only; the result lands in ``dev_result`` (16 device bytes)."""
+        _check(lib().fsm_run_spec_k_async(self._h, _ptr(inp), length, k, _ptr(dev_result)),
+               "fsm_run_spec_k_async")
+
+    def run_spec_k_host(self, host_inp, length: int, k: int) -> tuple[int, int]:
+        """fsm_run_spec_k_host: end-to-end over a host buffer (numpy array / pinned tensor)."""
+        q, n = _U32(), _U64()
+        _check(lib().fsm_run_spec_k_host(self._h, _ptr(host_inp), length, k, ctypes.byref(q), ctypes.byref(n)),
+               "fsm_run_spec_k_host")
+        return int(q.value), int(n.value)
+
+    def run_shard(self, inp, length: int, halo=None, halo_len: int = 0, k: int = 1, keep: bool = False):
+        """fsm_run_shard -> (fsm_shard_map, shard handle or None)."""
+        m = fsm_shard_map()
+        st = _P()
+        _check(lib().fsm_run_shard(self._h, _ptr(inp), length, _ptr(halo) if halo is not None else None,
+                                   halo_len, k, ctypes.byref(m), ctypes.byref(st) if keep else None),
+               "fsm_run_shard")
+        return m, (Shard(st) if keep else None)
+
+    def shard_fixup(self, shard: "Shard", true_start: int) -> tuple[int, int]:
+        q, n = _U32(), _U64()
+        _check(lib().fsm_shard_fixup(self._h, shard._h, true_start, ctypes.byref(q), ctypes.byref(n)),
+               "fsm_shard_fixup")
+        return int(q.value), int(n.value)
+
+
+class Shard:
+    def __init__(self, h):
+        self._h = h
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().fsm_shard_free(self._h)
+            self._h = None
+
+    __del__ = close

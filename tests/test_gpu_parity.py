@@ -1,0 +1,235 @@
+"""GPU parity: the CUDA path (through the C ABI) against the sequential oracle, bit-exact in the
+final state and the accept count, on seeded synthetic DFAs and inputs that span
+several tiles and a ragged tail, every table variant, every instantiated k, both merges, the
+async / host-buffer / shard entry points, and the edge cases (empty input, unaligned pointers,
+bit-mode tails, out-of-alphabet bytes, k = N, k > |image|)."""
+import numpy as np
+import pytest
+
+from fsmgen import dfas, streams
+from oracle import seq, speck
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from paper_conf_ppopp_xiaja20_b200 import fsmspec  # noqa: E402
+from paper_conf_ppopp_xiaja20_b200.fsmspec import FSM  # noqa: E402
+
+
+def dev(data: np.ndarray, offset: int = 0):
+    buf = torch.zeros(data.size + offset + 64, dtype=torch.uint8, device="cuda")
+    buf[offset:offset + data.size] = torch.from_numpy(np.ascontiguousarray(data))
+    return buf, buf.data_ptr() + offset
+
+
+def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
+    if length is None:
+        length = data.size * 8 if dfa.bit_mode else data.size
+    with FSM.from_dfa(dfa) as f:
+        if opt:
+            f.set_options(**opt)
+        buf, ptr = dev(data, offset)
+        res = f.run_spec_k(ptr, length, k)
+        st = f.stats()
+        torch.cuda.synchronize()
+    return res, st
+
+
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3}
+
+
+def fits(dfa, var):
+    n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
+    return {"P4": n <= 4, "P8": n <= 8, "B": n <= 256, "G": True}[var]
+
+
+# --------------------------------------------------------------------- worked example on GPU
+@pytest.mark.parametrize("var", ["P4", "P8", "B", "G"])
+@pytest.mark.parametrize("k", [1, 2, 3, 4])
+def test_fig1_worked_example(var, k):
+    d = dfas.c_comment(True)
+    data = np.frombuffer(b"/*xxx**/", np.uint8)
+    (q, n), _ = gpu_run(d, data, k=k, variant=VARIANTS[var])
+    assert (q, n) == (0, 1) == seq.run(d, data)
+
+
+# --------------------------------------------------------------------- C1-shaped text
+@pytest.mark.parametrize("var", ["P4", "P8", "B", "G"])
+@pytest.mark.parametrize("chunk", [0, 64, 96, 4096])
+def test_c_comment_text(var, chunk):
+    d = dfas.c_comment(True)
+    data = streams.c_source(300_001, seed=streams.MASTER_SEED + 1, comment_frac=0.3)
+    exp = seq.run(d, data)
+    for k in (1, 2, 4):
+        got, st = gpu_run(d, data, k=k, variant=VARIANTS[var], chunk_bytes=chunk)
+        assert got == exp, (var, chunk, k, st)
+
+
+# --------------------------------------------------------------------- random DFAs, all variants, all k
+CASES = [(2, 2), (4, 2), (4, 4), (7, 3), (8, 1), (8, 2), (8, 8), (16, 2), (16, 5), (100, 4), (255, 8),
+         (1000, 3), (4096, 8)]
+
+
+@pytest.mark.parametrize("n,m", CASES)
+def test_random_dfa_parity(n, m):
+    d = dfas.random_dfa(n, m, seed=1000 + n * 17 + m)
+    length = 1_000_003
+    data = streams.splitmix_bytes(5 + n, 0, length)
+    exp = seq.run(d, data)
+    for var in VARIANTS:
+        if not fits(d, var):
+            continue
+        for k in sorted({1, 2, 3, min(m, 16), min(n, 16), 5, 16} & set(range(1, min(n, 16) + 1))):
+            for chunk in (64, 1024):
+                got, st = gpu_run(d, data, k=k, variant=VARIANTS[var], chunk_bytes=chunk)
+                assert got == exp, (n, m, var, k, chunk, st)
+                if k >= m:
+                    assert st["reexec_chunks"] == 0, st  # k >= |image| never re-executes
+
+
+@pytest.mark.parametrize("length", [0, 1, 2, 31, 32, 33, 63, 64, 65, 4095, 4096, 4097, 65536 * 3 + 7])
+@pytest.mark.parametrize("offset", [0, 1, 13, 32])
+def test_lengths_and_alignment(length, offset):
+    d = dfas.random_dfa(8, 3, seed=42)
+    data = streams.splitmix_bytes(77, 0, max(length, 1))[:length]
+    exp = seq.run(d, data, length)
+    for k in (1, 2, 3):
+        got, _ = gpu_run(d, data, length, k=k, offset=offset, chunk_bytes=64)
+        assert got == exp, (length, offset, k)
+
+
+def test_out_of_alphabet_is_reported():
+    d = dfas.c_comment(False)   # 3-symbol alphabet -> internal sink
+    good = np.array([0, 1, 2, 2, 1, 0] * 5000, np.uint8)
+    assert gpu_run(d, good, k=2)[0] == seq.run(d, good)
+    bad = good.copy()
+    bad[12345] = 7
+    with pytest.raises(fsmspec.SymbolError):
+        gpu_run(d, bad, k=2)
+
+
+# --------------------------------------------------------------------- bit mode (Huffman, Div7)
+@pytest.mark.parametrize("n_bits", [0, 1, 3, 8, 13, 4096 * 8 + 5, 1_000_003])
+def test_div7_bits(n_bits):
+    d = dfas.div7()
+    data = streams.random_bits(max(n_bits, 1), seed=n_bits)
+    exp = seq.run(d, data, n_bits)
+    for k in (1, 3, 7):
+        for var in ("P8", "B", "G"):
+            got, st = gpu_run(d, data, n_bits, k=k, variant=VARIANTS[var], chunk_bytes=64)
+            assert got == exp, (n_bits, k, var)
+            if k == 7:
+                assert st["reexec_chunks"] == 0   # spec-N
+
+
+def test_div7_closed_form_on_gpu():
+    d = dfas.div7()
+    n_bits = 5000
+    data = streams.random_bits(n_bits, seed=3)
+    bits = "".join(str(b) for b in seq.bits_of(data, n_bits))
+    got, _ = gpu_run(d, data, n_bits, k=7)
+    assert got[0] == int(bits, 2) % 7
+
+
+def test_huffman_zipf():
+    w = dfas.zipf_weights(256, seed=streams.MASTER_SEED + 2)
+    d, codes = dfas.huffman(w.tolist())
+    n_bits = 3_000_005
+    data, nsym = streams.huffman_bits(codes, w / w.sum(), n_bits, seed=11)
+    exp = seq.run(d, data, n_bits)
+    assert exp[1] == nsym
+    for k in (1, 2, 4):
+        for var in ("B", "G"):
+            got, st = gpu_run(d, data, n_bits, k=k, variant=VARIANTS[var])
+            assert got == exp, (k, var, st)
+
+
+def test_aho_corasick():
+    pats = dfas.snort_patterns(1024, seed=streams.MASTER_SEED + 3)
+    d = dfas.aho_corasick(pats)
+    rng = np.random.default_rng(3)
+    data = rng.integers(0, 256, 2_000_000).astype(np.uint8)
+    for _ in range(500):
+        p = pats[int(rng.integers(0, len(pats)))]
+        pos = int(rng.integers(0, data.size - len(p)))
+        data[pos:pos + len(p)] = np.frombuffer(p, np.uint8)
+    exp = seq.run(d, data)
+    for k in (1, 2, 4):
+        got, _ = gpu_run(d, data, k=k)
+        assert got == exp
+
+
+# --------------------------------------------------------------------- other entry points
+def test_sequential_merge_ablation_parity():
+    d = dfas.random_dfa(16, 5, seed=9)
+    data = streams.splitmix_bytes(9, 0, 2_000_017)
+    exp = seq.run(d, data)
+    for k in (1, 2, 5):
+        got, st = gpu_run(d, data, k=k, merge=fsmspec.FSM_MERGE_SEQUENTIAL)
+        assert got == exp, (k, st)
+    got, st = gpu_run(dfas.div7(), streams.random_bits(100_000, 1), 100_000, k=3,
+                      merge=fsmspec.FSM_MERGE_SEQUENTIAL, chunk_bytes=64)
+    assert got == seq.run(dfas.div7(), streams.random_bits(100_000, 1), 100_000)
+
+
+def test_async_and_host_entry_points():
+    d = dfas.random_dfa(8, 2, seed=5)
+    data = streams.splitmix_bytes(21, 0, 5_000_000)
+    exp = seq.run(d, data)
+    with FSM.from_dfa(d) as f:
+        buf, ptr = dev(data)
+        res = torch.zeros(4, dtype=torch.int32, device="cuda")
+        f.run_spec_k_async(ptr, data.size, 2, res.data_ptr())
+        r = res.cpu().numpy().view(np.uint32)
+        assert (int(r[0]), int(r[2]) | (int(r[3]) << 32)) == exp
+        assert f.run_spec_k_host(data, data.size, 2) == exp
+        pinned = torch.from_numpy(data).pin_memory()
+        assert f.run_spec_k_host(pinned.data_ptr(), data.size, 1) == exp
+
+
+def test_host_entry_point_multi_piece():
+    d = dfas.random_dfa(16, 3, seed=6)
+    length = (1 << 28) + 12345   # two 256 MiB pieces chained on the device
+    data = np.empty(length, np.uint8)
+    streams.splitmix_bytes(31, 0, length, out=data)
+    exp = seq.run(d, data)
+    with FSM.from_dfa(d) as f:
+        assert f.run_spec_k_host(data, length, 3) == exp
+
+
+# --------------------------------------------------------------------- shards (multi-GPU logic)
+@pytest.mark.parametrize("G", [2, 3, 5])
+@pytest.mark.parametrize("k", [1, 2])
+def test_shard_maps_compose_and_fixup(G, k):
+    """Single-GPU emulation of G shards: per-shard maps keyed on the halo's
+    look-back set equal the oracle from each start; composing them and fixing up the
+    shard-boundary misses gives the oracle result."""
+    d = dfas.random_dfa(16, 4, seed=77 + G)
+    L = 3_000_000
+    data = streams.splitmix_bytes(4 + G, 0, L)
+    exp = seq.run(d, data)
+    bounds = [L * g // G // 32 * 32 for g in range(G)] + [L]
+    buf, base = dev(data)
+    with FSM.from_dfa(d) as f:
+        maps, shards = [], []
+        for g in range(G):
+            lo, hi = bounds[g], bounds[g + 1]
+            m, st = f.run_shard(base + lo, hi - lo, halo=(base + lo - 1) if g else None,
+                                halo_len=1 if g else 0, k=k, keep=True)
+            # each slot equals the oracle run from its start
+            for s, e, c in m.slots():
+                assert (e, c) == seq.run_from(d, s, data[lo:hi]), (g, s)
+            if g:
+                starts = [s for s, _, _ in m.slots()]
+                assert starts == speck.lookback(d.table, int(data[lo - 1]), k)
+            maps.append(m)
+            shards.append(st)
+        x, total = d.start, 0
+        for g in range(G):
+            hit = [(e, c) for s, e, c in maps[g].slots() if s == x]
+            if hit:
+                e, c = hit[0]
+            else:
+                e, c = f.shard_fixup(shards[g], x)
+            x, total = e, total + c
+        assert (x, total) == exp

@@ -253,7 +253,7 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
     const uint32_t n = f->dfa.n;
     f->auto_variant = n <= 4 ? VAR_P4 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B : VAR_G;
     f->opt.chunk_bytes = 0;
-    f->opt.threads_per_tile = kThreads;
+    f->opt.threads_per_tile = 0;  // auto: max_threads(K)
     f->opt.variant = FSM_VARIANT_AUTO;
     f->opt.merge = FSM_MERGE_PARALLEL;
     f->opt.ctas_per_sm = 0;
@@ -329,14 +329,15 @@ extern "C" int fsm_set_stream(fsm_t *f, void *s)
 extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
 {
     if (!f || !o) return FSM_EINVAL;
-    if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > (1u << 24))) return FSM_EINVAL;
-    if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > kThreads))
+    // chunk <= 8 KiB keeps 32-tile look-back windows of counts inside 32 bits (8 per byte in bit mode)
+    if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
+    if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
     if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_G) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
-    f->opt.chunk_bytes = o->chunk_bytes;  // 0 = adaptive
-    if (o->threads_per_tile) f->opt.threads_per_tile = o->threads_per_tile;
+    f->opt.chunk_bytes = o->chunk_bytes;            // 0 = adaptive
+    f->opt.threads_per_tile = o->threads_per_tile;  // 0 = auto
     f->opt.variant = o->variant;
     f->opt.merge = o->merge;
     f->opt.ctas_per_sm = o->ctas_per_sm;
@@ -377,14 +378,23 @@ static int variant_of(const fsm *f, int force)
     return f->opt.variant == FSM_VARIANT_AUTO ? f->auto_variant : f->opt.variant;
 }
 
-static uint32_t pick_chunk(const fsm *f, uint64_t len_bytes, uint32_t T)
+// Geometry: T chunks per tile (CTA threads), chunk bytes.  Large inputs: the largest CTA the
+// register budget allows for K and 4 KiB chunks.  Small inputs: shrink the CTA, then the chunk,
+// so that every SM still gets a few tiles.
+static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, uint32_t &T, uint32_t &chunk)
 {
-    if (f->opt.chunk_bytes) return f->opt.chunk_bytes;
-    // enough chunks to give every SM several resident tiles, chunks of 64 B .. 4 KiB
+    const uint32_t tmax = (uint32_t)max_threads(K);
+    T = f->opt.threads_per_tile ? std::min<uint32_t>(f->opt.threads_per_tile, tmax) : tmax;
+    if (!f->opt.threads_per_tile)
+        while (T > 128 && len_bytes < (uint64_t)f->num_sms * T * 4096) T >>= 1;
+    if (f->opt.chunk_bytes) {
+        chunk = f->opt.chunk_bytes;
+        return;
+    }
     const uint64_t want_chunks = (uint64_t)f->num_sms * 2 * T;
     uint64_t c = (len_bytes + want_chunks - 1) / want_chunks;
     c = (c + 31) & ~31ull;
-    return (uint32_t)std::min<uint64_t>(4096, std::max<uint64_t>(64, c));
+    chunk = (uint32_t)std::min<uint64_t>(4096, std::max<uint64_t>(64, c));
 }
 
 static int ensure_desc(fsm *f, size_t ntiles)
@@ -407,10 +417,11 @@ static int launch_run(fsm *f, const RunSpec &r)
 {
     const int var = variant_of(f, r.force_variant);
     const int K = kslots(r.k);
-    const uint32_t T = f->opt.threads_per_tile;
     const bool bits = f->mode == FSM_INPUT_BITS_MSB;
     const uint64_t len_bytes = bits ? r.len_sym / 8 : r.len_sym;
-    const uint32_t chunk = pick_chunk(f, len_bytes, T);
+    uint32_t T = 0, chunk = 0;
+    pick_geometry(f, len_bytes, K, T, chunk);
+    if (r.merge == FSM_MERGE_SEQUENTIAL) T = std::min<uint32_t>(T, kThreads);
     const uint64_t tile_bytes = (uint64_t)T * chunk;
     uint64_t ntiles64 = (len_bytes + tile_bytes - 1) / tile_bytes;
     if (ntiles64 == 0) ntiles64 = 1;

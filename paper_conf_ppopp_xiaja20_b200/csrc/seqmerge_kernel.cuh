@@ -73,7 +73,7 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
     const uint64_t nbatch = (nch + T - 1) / T;
     auto load = [&](uint64_t batch, int buf) {
         const uint64_t g0 = batch * T;
-        for (uint32_t i = threadIdx.x; i < T * K; i += T) {
+        for (uint32_t i = threadIdx.x - 1; i < T * K; i += T - 1) {  // threads 1..T-1
             const uint64_t g = g0 + i / K;
             if (g < nch) {
                 bS[buf * T * K + i] = sb.S[g0 * K + i];

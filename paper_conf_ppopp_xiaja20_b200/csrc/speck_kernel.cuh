@@ -28,7 +28,11 @@
 namespace speck {
 
 enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3 };
-constexpr int kThreads = 256;
+constexpr int kThreads = 256;  // auxiliary kernels
+// Threads per tile (one chunk per thread) of the fused kernel, by the number of chains K: large
+// CTAs keep few tiles in flight (short look-back windows) at one CTA per SM; the register budget
+// caps them for large K.
+__host__ __device__ constexpr int max_threads(int K) { return K <= 3 ? 1024 : K <= 6 ? 512 : 256; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
 
 // ------------------------------------------------------------------------------- PTX helpers --
@@ -59,6 +63,16 @@ __device__ __forceinline__ Bytes32 ldg256(const uint8_t *p)
 __device__ __forceinline__ uint4 ldg128(const uint8_t *p)
 {
     return __ldg(reinterpret_cast<const uint4 *>(p));
+}
+
+// PTX prmt in its default mode: every selector nibble is used as-is.  CUDA's __byte_perm masks
+// the selector with 0x7777 first (an extra LOP3 on the dependency chain); the packed variants
+// keep bit 3 of the low nibble zero by construction and ignore result bytes 1-3.
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel)
+{
+    uint32_t d;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(sel));
+    return d;
 }
 
 // ------------------------------------------------------------------- table-placement variants --
@@ -104,19 +118,19 @@ struct TablePacked {
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
     {
         // address = c * 256 + lane * 4|8, built by one PRMT: byte1 <- byte j of w, byte0 <- lanereg
-        const uint32_t a = __byte_perm(w, lanereg, 0x5504u | (uint32_t(j) << 4));
+        const uint32_t a = prmt(w, lanereg, 0x5504u | (uint32_t(j) << 4));
         if (kWide) {
             const uint2 r = *reinterpret_cast<const uint2 *>(sm + a);
 #pragma unroll
             for (int s = 0; s < K; s++) {
-                cur[s] = __byte_perm(r.x, r.y, cur[s]);
+                cur[s] = prmt(r.x, r.y, cur[s]);
                 acc[s] += cur[s] & 0xF0u;
             }
         } else {
             const uint32_t r = *reinterpret_cast<const uint32_t *>(sm + a);
 #pragma unroll
             for (int s = 0; s < K; s++) {
-                cur[s] = __byte_perm(r, 0u, cur[s]);
+                cur[s] = prmt(r, 0u, cur[s]);
                 acc[s] += cur[s] & 0xF0u;
             }
         }
@@ -129,7 +143,7 @@ struct TablePacked {
     }
     __device__ __forceinline__ uint32_t apply(Row r, uint32_t st, uint32_t &cnt) const
     {
-        const uint32_t f = __byte_perm(r.x, r.y, st) & 0xFFu;
+        const uint32_t f = prmt(r.x, r.y, st) & 0xFFu;
         cnt += f >> 4;
         return f & 0xFu;
     }
@@ -419,7 +433,7 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
 
 // ------------------------------------------------------------------------------- the kernel --
 template <int K, int VAR>
-__global__ void __launch_bounds__(kThreads) speck_kernel(Params p)
+__global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
 {
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
@@ -577,20 +591,19 @@ __global__ void __launch_bounds__(kThreads) speck_kernel(Params p)
         }
         __syncwarp();
 
-        // a7: publish the aggregate A_b
+        // a7: publish the aggregate A_b (slot = {start, end, count})
         TileDesc *D = p.desc + tile;
         if (lane < K) {
             const uint32_t sv = Sj[lane];
-            D->astart[lane] = sv == 0xFFFFu ? NOSTATE : sv;
-            D->aend[lane] = Qe[lane] & 0xFFFFu;
-            D->acnt[lane] = Qc[lane];
+            D->aslot[lane] = make_uint4(sv == 0xFFFFu ? NOSTATE : sv, Qe[lane] & 0xFFFFu, Qc[lane], 0u);
         }
         __threadfence();
         __syncwarp();
         const uint32_t ep = p.epoch << 2;
         if (lane == 0) st_release(&D->flag, ep | ST_A);
 
-        // a7: decoupled look-back -> exclusive prefix E (lane s = shard slot s)
+        // a7: decoupled look-back -> exclusive prefix E (lane s holds shard slot s).
+        // (1) walk back 32 descriptors at a time to the nearest inclusive prefix P_m.
         uint32_t Es = 0;
         unsigned long long Ec = 0;
         bool Ev = false;
@@ -609,7 +622,7 @@ __global__ void __launch_bounds__(kThreads) speck_kernel(Params p)
                 const int fp = pm ? __ffs(pm) - 1 : 32;
                 const unsigned before = fp >= 32 ? 0xFFFFFFFFu : ((1u << fp) - 1u);
                 if (xm & before) {
-                    __nanosleep(100);
+                    __nanosleep(64);
                     continue;
                 }
                 if (fp < 32) {
@@ -644,29 +657,60 @@ __global__ void __launch_bounds__(kThreads) speck_kernel(Params p)
         } else {
             load_P(m);
         }
-        for (int64_t tt = m + 1; tt < (int64_t)tile; tt++) {
-            const TileDesc *Dt = p.desc + tt;
-            const uint32_t f0 = __shfl_sync(0xFFFFFFFFu, ld_acquire(&Dt->flag), 0);
-            if ((f0 & 3u) == ST_P) {
-                load_P(tt);
-                continue;
-            }
-            // each lane acquires for itself before reading the A payload
-            while ((ld_acquire(&Dt->flag) & ~3u) != ep) __nanosleep(32);
-            bool hit = false;
-            if (Ev) {
-#pragma unroll 4
+        // (2) apply the aggregates A_{m+1} .. A_{b-1}, 32 per step: every lane loads one tile's
+        // aggregate in parallel, a warp suffix scan composes the 32 mappings (the same operator as
+        // the chunk merge), and the composed window is applied to E.  A slot that breaks inside the
+        // window hit a tile-boundary miss there: take that tile's P and continue after it.
+        for (int64_t nx = m + 1; nx < (int64_t)tile;) {
+            const int64_t tt = nx + lane;
+            uint32_t S2[K], e2[K], c2[K];
+            bool id2 = tt >= (int64_t)tile;
+            if (!id2) {
+                const TileDesc *Dt = p.desc + tt;
+                while ((ld_acquire(&Dt->flag) & ~3u) != ep) __nanosleep(32);
+#pragma unroll
                 for (int l = 0; l < K; l++) {
-                    if (__ldcg(&Dt->astart[l]) == Es) {
-                        const uint32_t ne = __ldcg(&Dt->aend[l]);
-                        Ec += __ldcg(&Dt->acnt[l]);
-                        Es = ne;
-                        hit = true;
-                        break;
+                    const uint4 v = __ldcg(&Dt->aslot[l]);
+                    S2[l] = v.x;
+                    e2[l] = v.x == NOSTATE ? (ABSENT << 16) : (v.y | (COMPLETE << 16));
+                    c2[l] = v.z;
+                }
+            } else {
+#pragma unroll
+                for (int l = 0; l < K; l++) S2[l] = NOSTATE, e2[l] = ABSENT << 16, c2[l] = 0;
+            }
+            warp_suffix_scan<K>(S2, e2, c2, id2, 0, 1);
+            int brk = 32;
+            {
+                uint32_t ne = 0, nc = 0;
+                bool found = false;
+#pragma unroll
+                for (int l = 0; l < K; l++) {
+                    const uint32_t sl = __shfl_sync(0xFFFFFFFFu, S2[l], 0);
+                    const uint32_t el = __shfl_sync(0xFFFFFFFFu, e2[l], 0);
+                    const uint32_t cl = __shfl_sync(0xFFFFFFFFu, c2[l], 0);
+                    if (Ev && sl == Es) {
+                        ne = el;
+                        nc = cl;
+                        found = true;
+                    }
+                }
+                if (Ev) {
+                    if (!found) brk = 0;
+                    else if ((ne >> 16) != COMPLETE) brk = (int)(ne >> 16);
+                    else {
+                        Es = ne & 0xFFFFu;
+                        Ec += nc;
                     }
                 }
             }
-            if (__ballot_sync(0xFFFFFFFFu, Ev && !hit)) load_P(tt);  // a tile-boundary miss upstream
+            const int mb = __reduce_min_sync(0xFFFFFFFFu, brk);
+            if (mb < 32) {
+                load_P(nx + mb);  // E := P of the tile where a slot broke (it resolves its own miss)
+                nx = nx + mb + 1;
+            } else {
+                nx += 32;
+            }
         }
 
         // own inclusive prefix P_b = E then A_b; a tile-boundary miss resolves through chunk 0.

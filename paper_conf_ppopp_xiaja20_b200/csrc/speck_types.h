@@ -25,9 +25,8 @@ enum Status : uint32_t { ST_X = 0, ST_A = 1, ST_P = 2 };
 struct __align__(128) TileDesc {
     uint32_t flag;                 // epoch << 2 | Status
     uint32_t pmask;                // P: valid slots
-    uint32_t astart[KMAX];         // A: start set of the tile's first chunk (NOSTATE = absent)
-    uint32_t aend[KMAX];           // A: end state per slot (ABSENT slots: unspecified)
-    uint32_t acnt[KMAX];           // A: accept count per slot within the tile
+    uint32_t pad[2];
+    uint4 aslot[KMAX];             // A: {start (NOSTATE = absent), end, count within tile, 0}
     uint32_t pstate[KMAX];         // P: state after this tile, per shard slot
     unsigned long long pcnt[KMAX]; // P: count up to and including this tile, per shard slot
 };

@@ -156,9 +156,9 @@ class FSM:
         return cls(dfa.table, dfa.start, dfa.accept, dfa.bit_mode)
 
     def close(self) -> None:
-        if getattr(self, "_h", None):
-            lib().fsm_destroy(self._h)
-            self._h = None
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.fsm_destroy(self._h)
+        self._h = None
 
     __del__ = close
 
@@ -229,8 +229,8 @@ class Shard:
         self._h = h
 
     def close(self):
-        if getattr(self, "_h", None):
-            lib().fsm_shard_free(self._h)
-            self._h = None
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.fsm_shard_free(self._h)
+        self._h = None
 
     __del__ = close

@@ -48,7 +48,16 @@ def make_workload(args):
             streams.splitmix_fill_device(ptr, sseed, lo, n, stream)
 
         def host(lo, n, out=None):
-            return streams.splitmix_bytes(sseed, lo, n, out=out)
+            # multi-threaded host regeneration of the same counter-based stream
+            import concurrent.futures as cf
+
+            if out is None:
+                out = np.empty(n, dtype=np.uint8)
+            piece = 1 << 28
+            with cf.ThreadPoolExecutor(os.cpu_count()) as ex:
+                list(ex.map(lambda o: streams.splitmix_bytes(sseed, lo + o, min(piece, n - o), out=out[o:]),
+                            range(0, n, piece)))
+            return out[:n]
 
         name = (f"C5 random DFA N={args.n_states} m={args.m} (|image(c)|=m), spec-{args.k}, "
                 f"{args.size_gib:g} GiB i.i.d. bytes")

@@ -22,6 +22,7 @@ struct FixParams {
     uint32_t end[KMAX];
     unsigned long long count[KMAX];
     unsigned long long *out;   // [0] = converged flag, [1] = end, [2] = count, [3] = bytes consumed
+    KConst kc;
 };
 
 template <int VAR>
@@ -30,7 +31,7 @@ __global__ void __launch_bounds__(kThreads) fixup_kernel(FixParams f)
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
     TB tb;
-    tb.setup(smem, f.table, f.n_states);
+    tb.setup(smem, f.table, f.n_states, f.kc);
     __syncthreads();
     if (threadIdx.x != 0) return;
     uint32_t y[KMAX], cy[KMAX];

@@ -450,6 +450,9 @@ static int launch_run(fsm *f, const RunSpec &r)
     p.result = r.result;
     p.stats = f->d_stats;
     p.ticket = f->d_ticket;
+    p.k_1e24 = 1u << 24;
+    p.k_16 = 16;
+    p.k_512 = 512;
 
     const size_t smem = Layout(T, K, p.table_bytes).total;
 
@@ -700,6 +703,7 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         fp.count[s] = st->map.count[s];
     }
     fp.out = f->d_fix;
+    fp.kc = KConst{1u << 24, 16, 512};
     FixFn fn = get_fix(var);
     const size_t smem = std::max<uint32_t>(16, f->img_bytes[var]);
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

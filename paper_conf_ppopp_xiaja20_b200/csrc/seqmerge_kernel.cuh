@@ -24,7 +24,7 @@ __global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
     TB tb;
-    tb.setup(smem, p.table, p.n_states);
+    tb.setup(smem, p.table, p.n_states, kconst(p));
     __syncthreads();
     const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
     const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
@@ -40,18 +40,19 @@ __global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb
 #pragma unroll
             for (int s = 0; s < K; s++) S[s] = (uint32_t)s < ni ? (uint32_t)__ldg(p.lb + c * KMAX + s) : NOSTATE;
         }
-        uint32_t cur[K], acc[K];
+        uint32_t cur[K], acc[K], accf[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
-            cur[s] = tb.init(S[s] == NOSTATE ? 0u : S[s]);
+            cur[s] = tb.init(S[s] == NOSTATE ? (S[0] == NOSTATE ? 0u : S[0]) : S[s]);
             acc[s] = 0;
+            accf[s] = 0;
         }
-        if (e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc);
+        if (e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf);
 #pragma unroll
         for (int s = 0; s < K; s++) {
             sb.S[g * K + s] = (uint16_t)(S[s] == NOSTATE ? 0xFFFFu : S[s]);
             sb.E[g * K + s] = tb.state_of(cur[s]);
-            sb.C[g * K + s] = tb.count_of(acc[s]);
+            sb.C[g * K + s] = tb.count_of(acc[s], accf[s]);
         }
     }
 }
@@ -62,7 +63,7 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
     TB tb;
-    tb.setup(smem, p.table, p.n_states);
+    tb.setup(smem, p.table, p.n_states, kconst(p));
     const uint32_t T = blockDim.x;
     const uint32_t tb_bytes = (p.table_bytes + 15) & ~15u;
     // double-buffered batches of T mappings

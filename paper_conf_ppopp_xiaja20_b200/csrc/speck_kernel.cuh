@@ -60,6 +60,37 @@ __device__ __forceinline__ Bytes32 ldg256(const uint8_t *p)
                  : "l"(p));
     return r;
 }
+// Same load with an L2 fetch-size hint: the L2 pulls 256 B from DRAM, so the lane's next seven
+// 32-byte blocks arrive from L2 instead of HBM (deeper effective prefetch without registers).
+__device__ __forceinline__ Bytes32 ldg256_l2pf(const uint8_t *p)
+{
+    Bytes32 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.w[0]), "=r"(r.w[1]), "=r"(r.w[2]), "=r"(r.w[3]), "=r"(r.w[4]), "=r"(r.w[5]),
+                   "=r"(r.w[6]), "=r"(r.w[7])
+                 : "l"(p));
+    return r;
+}
+__device__ __forceinline__ void prefetch_l2(const uint8_t *p)
+{
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+#ifndef FSM_LOADMODE
+#define FSM_LOADMODE 0
+#endif
+// streaming load of block i of the chunk (FSM_LOADMODE 0: plain, 1: L2::256B hint, 2: plain +
+// explicit L2 prefetch 8 blocks ahead)
+__device__ __forceinline__ Bytes32 ldg_block(const uint8_t *p, uint64_t i, uint64_t nblk)
+{
+#if FSM_LOADMODE == 1
+    return ldg256_l2pf(p + 32 * i);
+#elif FSM_LOADMODE == 2
+    if (i + 8 < nblk) prefetch_l2(p + 32 * (i + 8));
+    return ldg256(p + 32 * i);
+#else
+    return ldg256(p + 32 * i);
+#endif
+}
 __device__ __forceinline__ uint4 ldg128(const uint8_t *p)
 {
     return __ldg(reinterpret_cast<const uint4 *>(p));
@@ -74,6 +105,26 @@ __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel)
     asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(sel));
     return d;
 }
+
+// FMA-pipe integer helpers (IMAD / IMAD.HI).  The hot loop is ALU-pipe bound (PRMT, LOP3,
+// IADD3 all issue there); half of the accept-count work is moved to the otherwise idle FMA pipe.
+__device__ __forceinline__ uint32_t mad_hi(uint32_t a, uint32_t b, uint32_t c)
+{
+    uint32_t d;
+    asm("mad.hi.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+    return d;
+}
+__device__ __forceinline__ uint32_t mad_lo(uint32_t a, uint32_t b, uint32_t c)
+{
+    uint32_t d;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+    return d;
+}
+
+struct KConst {
+    uint32_t k_1e24, k_16, k_512;
+};
+__device__ __forceinline__ KConst kconst(const Params &p) { return KConst{p.k_1e24, p.k_16, p.k_512}; }
 
 // ------------------------------------------------------------------- table-placement variants --
 // Every variant exposes
@@ -92,10 +143,12 @@ struct TablePacked {
     static constexpr bool kWide = VAR == VAR_P8;
     const uint8_t *sm;
     uint32_t lanereg;
-    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t)
+    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t, const KConst &kc)
     {
         sm = s;
         lanereg = (threadIdx.x & 31) * (kWide ? 8 : 4);
+        c24 = kc.k_1e24;
+        c16 = kc.k_16;
         if (kWide) {
             const uint2 *rows = static_cast<const uint2 *>(g);
             for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
@@ -110,29 +163,31 @@ struct TablePacked {
             }
         }
     }
+    uint32_t c24, c16;  // 1 << 24 and 16 as opaque registers so that ptxas keeps IMAD / IMAD.HI (FMA pipe)
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur & 0xFu; }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc) const { return acc >> 4; }
+    // acc: count * 16 (ALU-pipe accumulation), accf: count (FMA-pipe accumulation)
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf) const { return (acc >> 4) + accf; }
 
     template <int K>
-    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
     {
         // address = c * 256 + lane * 4|8, built by one PRMT: byte1 <- byte j of w, byte0 <- lanereg
         const uint32_t a = prmt(w, lanereg, 0x5504u | (uint32_t(j) << 4));
+        uint32_t rx, ry = 0u;
         if (kWide) {
             const uint2 r = *reinterpret_cast<const uint2 *>(sm + a);
-#pragma unroll
-            for (int s = 0; s < K; s++) {
-                cur[s] = prmt(r.x, r.y, cur[s]);
-                acc[s] += cur[s] & 0xF0u;
-            }
+            rx = r.x;
+            ry = r.y;
         } else {
-            const uint32_t r = *reinterpret_cast<const uint32_t *>(sm + a);
+            rx = *reinterpret_cast<const uint32_t *>(sm + a);
+        }
 #pragma unroll
-            for (int s = 0; s < K; s++) {
-                cur[s] = prmt(r, 0u, cur[s]);
-                acc[s] += cur[s] & 0xF0u;
-            }
+        for (int s = 0; s < K; s++) {
+            cur[s] = prmt(rx, ry, cur[s]);                       // the chain: one PRMT per step
+            if (((j + s) & 1) == 0) acc[s] += cur[s] & 0xF0u;    // ALU: LOP3 (+ half an IADD3)
+            else accf[s] = mad_hi(cur[s] * c24, c16, accf[s]);   // FMA: IMAD, IMAD.HI (field >> 4)
         }
     }
     using Row = uint2;
@@ -152,26 +207,31 @@ struct TablePacked {
 // B: u16 entries T[s][c] = next | count << 8 in shared memory (N <= 256; 512 B per state).
 struct TableB {
     const uint8_t *sm;
-    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n)
+    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n, const KConst &kc)
     {
         sm = s;
+        c512 = kc.k_512;
+        c2e24 = kc.k_1e24;
         const uint4 *src = static_cast<const uint4 *>(g);
         uint4 *dst = reinterpret_cast<uint4 *>(s);
         for (uint32_t i = threadIdx.x; i < n * 32; i += blockDim.x) dst[i] = __ldg(src + i);
     }
+    uint32_t c512, c2e24;
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc) const { return acc >> 8; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf) const { return acc + accf; }
     template <int K>
-    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
     {
         const uint32_t c2 = j == 0 ? ((w << 1) & 0x1FEu) : ((w >> (8 * j - 1)) & 0x1FEu);
+        const uint8_t *base = sm + c2;
 #pragma unroll
         for (int s = 0; s < K; s++) {
-            const uint32_t e = *reinterpret_cast<const uint16_t *>(sm + (cur[s] << 9) + c2);
-            const uint32_t nx = e & 0xFFu;
-            acc[s] += e - nx;
-            cur[s] = nx;
+            // entry = next | count << 8; address = next * 512 + 2c on the FMA pipe (IMAD)
+            const uint32_t e = *reinterpret_cast<const uint16_t *>(base + mad_lo(cur[s], c512, 0u));
+            cur[s] = e & 0xFFu;
+            accf[s] = mad_hi(e, c2e24, accf[s]);  // + (e >> 8), FMA pipe
         }
     }
     using Row = uint32_t;
@@ -187,18 +247,19 @@ struct TableB {
 // G: u32 entries T[s][c] = next | count << 16 in global memory (L2-resident), any N <= 65535.
 struct TableG {
     const uint32_t *gt;
-    __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t) { gt = static_cast<const uint32_t *>(g); }
+    __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &) { gt = static_cast<const uint32_t *>(g); }
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc) const { return acc; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf) const { return acc + accf; }
     template <int K>
-    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
     {
         const uint32_t c = (w >> (8 * j)) & 0xFFu;
 #pragma unroll
         for (int s = 0; s < K; s++) {
             const uint32_t e = __ldg(gt + ((cur[s] << 8) | c));
-            acc[s] += e >> 16;
+            accf[s] = mad_hi(e, 1u << 16, accf[s]);  // + (e >> 16)
             cur[s] = e & 0xFFFFu;
         }
     }
@@ -220,13 +281,14 @@ template <> struct TableFor<VAR_G> { using type = TableG; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <int K, class TB>
-__device__ __forceinline__ void process32(const TB &tb, const Bytes32 &x, uint32_t (&cur)[K], uint32_t (&acc)[K])
+__device__ __forceinline__ void process32(const TB &tb, const Bytes32 &x, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                          uint32_t (&accf)[K])
 {
     if constexpr (K <= 4) {
 #pragma unroll
         for (int q = 0; q < 8; q++)
 #pragma unroll
-            for (int j = 0; j < 4; j++) tb.template step<K>(x.w[q], j, cur, acc);
+            for (int j = 0; j < 4; j++) tb.template step<K>(x.w[q], j, cur, acc, accf);
     } else {
         uint32_t w[8];
 #pragma unroll
@@ -234,36 +296,101 @@ __device__ __forceinline__ void process32(const TB &tb, const Bytes32 &x, uint32
 #pragma unroll 1
         for (int q = 0; q < 8; q++) {
 #pragma unroll
-            for (int j = 0; j < 4; j++) tb.template step<K>(w[0], j, cur, acc);
+            for (int j = 0; j < 4; j++) tb.template step<K>(w[0], j, cur, acc, accf);
 #pragma unroll
             for (int r = 0; r < 7; r++) w[r] = w[r + 1];
         }
     }
 }
 
-// Alg. 3 over bytes [b, e) of the input: 32-byte blocks with two blocks in flight,
-// then the ragged tail byte by byte.
+template <int K, class TB>
+__device__ __forceinline__ bool chains_converged(const TB &tb, const uint32_t (&cur)[K])
+{
+    bool c = true;
+#pragma unroll
+    for (int s = 1; s < K; s++) c = c && tb.state_of(cur[s]) == tb.state_of(cur[0]);
+    return c;
+}
+
+// Alg. 3 over bytes [b, e) of the input: 32-byte blocks (one full sector per lane per
+// LDG.256) with two blocks in flight, then the ragged tail byte by byte.
+// Convergence: two chains that reach the same state stay identical for the rest of the chunk
+// (the state-convergence property of [18]).  After every block the warp votes; once all
+// chains of every active lane coincide the remainder runs ONE chain and its count increments
+// are added to every slot -- bit-identical to running all k chains.  Absent slots start as a copy
+// of slot 0 so they never block the vote (their results are ignored).
 template <int K, class TB>
 __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restrict__ in, uint64_t b, uint64_t e,
-                                            bool aligned, uint32_t (&cur)[K], uint32_t (&acc)[K])
+                                            bool aligned, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                            uint32_t (&accf)[K])
 {
     const uint8_t *p = in + b;
     const uint64_t n = e - b;
     const uint64_t nblk = aligned ? (n >> 5) : 0;
+    uint64_t i = 0;
+    bool single = false;
+    Bytes32 x0, x1;
     if (nblk) {
-        Bytes32 x0 = ldg256(p), x1 = x0;
-        if (nblk > 1) x1 = ldg256(p + 32);
-        for (uint64_t i = 0; i < nblk; i++) {
+        x0 = ldg_block(p, 0, nblk);
+        x1 = x0;
+        if (nblk > 1) x1 = ldg_block(p, 1, nblk);
+        // two blocks per iteration so the double buffer alternates registers instead of moving them
+        for (; i < nblk;) {
             Bytes32 x2 = x1;
-            if (i + 2 < nblk) x2 = ldg256(p + 32 * (i + 2));
-            process32<K>(tb, x0, cur, acc);
-            x0 = x1;
-            x1 = x2;
+            if (i + 2 < nblk) x2 = ldg_block(p, i + 2, nblk);
+            process32<K>(tb, x0, cur, acc, accf);
+            i++;
+            if constexpr (K > 1) {
+                if (__all_sync(__activemask(), chains_converged<K>(tb, cur))) {
+                    x0 = x1;
+                    x1 = x2;
+                    single = true;
+                    break;
+                }
+            }
+            if (i >= nblk) break;
+            Bytes32 x3 = x2;
+            if (i + 2 < nblk) x3 = ldg_block(p, i + 2, nblk);
+            process32<K>(tb, x1, cur, acc, accf);
+            i++;
+            x0 = x2;
+            x1 = x3;
+            if constexpr (K > 1) {
+                if (__all_sync(__activemask(), chains_converged<K>(tb, cur))) {
+                    single = true;
+                    break;
+                }
+            }
         }
     }
-    for (uint64_t i = nblk << 5; i < n; i++) {
-        const uint32_t c = __ldg(p + i);
-        tb.template step<K>(c, 0, cur, acc);
+    if constexpr (K > 1) {
+        if (single) {
+            uint32_t c1[1] = {cur[0]}, a1[1] = {0u}, f1[1] = {0u};
+            while (i < nblk) {
+                Bytes32 x2 = x1;
+                if (i + 2 < nblk) x2 = ldg_block(p, i + 2, nblk);
+                process32<1>(tb, x0, c1, a1, f1);
+                if (++i >= nblk) break;
+                Bytes32 x3 = x2;
+                if (i + 2 < nblk) x3 = ldg_block(p, i + 2, nblk);
+                process32<1>(tb, x1, c1, a1, f1);
+                ++i;
+                x0 = x2;
+                x1 = x3;
+            }
+            for (uint64_t t = nblk << 5; t < n; t++) tb.template step<1>(__ldg(p + t), 0, c1, a1, f1);
+#pragma unroll
+            for (int s = 0; s < K; s++) {
+                cur[s] = c1[0];
+                acc[s] += a1[0];
+                accf[s] += f1[0];
+            }
+            return;
+        }
+    }
+    for (uint64_t t = nblk << 5; t < n; t++) {
+        const uint32_t c = __ldg(p + t);
+        tb.template step<K>(c, 0, cur, acc, accf);
     }
 }
 
@@ -444,7 +571,7 @@ __global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
     const uint32_t j = threadIdx.x;
 
     TB tb;
-    tb.setup(smem, p.table, p.n_states);
+    tb.setup(smem, p.table, p.n_states, kconst(p));
     const Layout L(T, K, p.table_bytes);
     uint32_t *Qe = reinterpret_cast<uint32_t *>(smem + L.qe);
     uint32_t *Qc = reinterpret_cast<uint32_t *>(smem + L.qc);
@@ -486,18 +613,19 @@ __global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
         }
 
         // ---- a4: local processing
-        uint32_t cur[K], acc[K];
+        uint32_t cur[K], acc[K], accf[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
-            cur[s] = tb.init(S[s] == NOSTATE ? 0u : S[s]);
+            cur[s] = tb.init(S[s] == NOSTATE ? (S[0] == NOSTATE ? 0u : S[0]) : S[s]);
             acc[s] = 0;
+            accf[s] = 0;
         }
-        if (!empty && e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc);
+        if (!empty && e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf);
         uint32_t eob[K], cnt[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
             eob[s] = S[s] == NOSTATE ? (ABSENT << 16) : (tb.state_of(cur[s]) | (COMPLETE << 16));
-            cnt[s] = tb.count_of(acc[s]);
+            cnt[s] = tb.count_of(acc[s], accf[s]);
         }
         bool ident = empty;
 

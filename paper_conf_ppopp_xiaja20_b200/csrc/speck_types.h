@@ -77,6 +77,9 @@ struct Params {
     const uint32_t *bittab;        // [n_states][2]: next | acc << 16
     DevResult *result;
     DevStats *stats;
+    // constants passed at run time so that ptxas cannot strength-reduce the FMA-pipe IMADs into
+    // ALU-pipe shifts (the hot loop balances the two pipes): 1 << 24, 16, 512
+    uint32_t k_1e24, k_16, k_512;
 };
 
 }  // namespace speck

@@ -12,7 +12,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_HERE, "libfsmspec.so")
+SO_PATH = os.environ.get("FSMSPEC_SO") or os.path.join(_HERE, "libfsmspec.so")  # override: experiments only
 
 FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 FSM_INPUT_BYTES, FSM_INPUT_BITS_MSB = 0, 1

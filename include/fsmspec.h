@@ -49,7 +49,7 @@ enum { FSM_INPUT_BYTES = 0, FSM_INPUT_BITS_MSB = 1 };
 /* Table-placement variants; FSM_VARIANT_AUTO picks by state count. */
 enum {
     FSM_VARIANT_AUTO = -1,
-    FSM_VARIANT_P4 = 0,  /* N <= 4:   packed 4 x u8 row per symbol, lane-replicated smem, PRMT chain */
+    FSM_VARIANT_P4 = 0,  /* N <= 4 (byte mode): packed 4 x u8 row per symbol, lane-replicated smem, PRMT chain */
     FSM_VARIANT_P8 = 1,  /* N <= 8:   packed 8 x u8 row per symbol, lane-replicated smem, PRMT chain */
     FSM_VARIANT_B = 2,   /* N <= 256: u16 entries (next | count << 8) in shared memory            */
     FSM_VARIANT_G = 3    /* any N:    u32 entries (next | count << 16) in global memory / L2      */

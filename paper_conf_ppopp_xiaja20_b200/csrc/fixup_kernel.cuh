@@ -30,6 +30,7 @@ __global__ void __launch_bounds__(kThreads) fixup_kernel(FixParams f)
 {
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
+    check_smem_window(VAR, scratch_offset(VAR, 0));
     TB tb;
     tb.setup(smem, f.table, f.n_states, f.kc);
     __syncthreads();

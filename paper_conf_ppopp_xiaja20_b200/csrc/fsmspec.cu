@@ -251,7 +251,7 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
     f->nimg.resize(256);
     build_lookback(f->dfa, f->lb.data(), f->nimg.data());
     const uint32_t n = f->dfa.n;
-    f->auto_variant = n <= 4 ? VAR_P4 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B : VAR_G;
+    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B : VAR_G;
     f->opt.chunk_bytes = 0;
     f->opt.threads_per_tile = 0;  // auto: max_threads(K)
     f->opt.variant = FSM_VARIANT_AUTO;
@@ -265,15 +265,15 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         return r;
     };
     // every variant the DFA fits, so that tests can force any of them
-    if (n <= 4) {
+    if (n <= 4 && !bits) {  // P4's count encoding is byte-mode only (count 0/1)
         auto img = image_packed(f->dfa, false);
         if ((rc = upload(&f->d_img[VAR_P4], img.data(), img.size()))) return fail(rc);
-        f->img_bytes[VAR_P4] = kPackedTableBytes;
+        f->img_bytes[VAR_P4] = 0;  // packed tables live in a fixed shared-window slot (scratch_offset)
     }
     if (n <= 8) {
         auto img = image_packed(f->dfa, true);
         if ((rc = upload(&f->d_img[VAR_P8], img.data(), img.size()))) return fail(rc);
-        f->img_bytes[VAR_P8] = kPackedTableBytes;
+        f->img_bytes[VAR_P8] = 0;
     }
     if (n <= 256) {
         auto img = image_b(f->dfa);
@@ -454,7 +454,7 @@ static int launch_run(fsm *f, const RunSpec &r)
     p.k_16 = 16;
     p.k_512 = 512;
 
-    const size_t smem = Layout(T, K, p.table_bytes).total;
+    const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes)).total;
 
     if (r.merge == FSM_MERGE_SEQUENTIAL) {
         if (r.keyed) return FSM_EINVAL;
@@ -505,14 +505,14 @@ static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T)
     SeqLocalFn lf;
     SeqWalkFn wf;
     get_seq(var, K, lf, wf);
-    const size_t smem_l = (p.table_bytes + 15) & ~15u;
+    const size_t smem_l = scratch_offset(var, p.table_bytes);
     CK(cudaFuncSetAttribute((const void *)lf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(smem_l, 16)));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lf, (int)T, std::max<size_t>(smem_l, 16)));
     const uint64_t blocks = std::min<uint64_t>((nch + T - 1) / T, (uint64_t)std::max(occ, 1) * f->num_sms);
     lf<<<(uint32_t)blocks, T, std::max<size_t>(smem_l, 16), f->stream>>>(p, f->seq);
     CK(cudaGetLastError());
-    const size_t smem_w = seq_walk_smem(T, K, p.table_bytes);
+    const size_t smem_w = seq_walk_smem(T, K, var, p.table_bytes);
     CK(cudaFuncSetAttribute((const void *)wf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_w));
     wf<<<1, T, smem_w, f->stream>>>(p, f->seq);
     CK(cudaGetLastError());
@@ -705,7 +705,7 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
     fp.out = f->d_fix;
     fp.kc = KConst{1u << 24, 16, 512};
     FixFn fn = get_fix(var);
-    const size_t smem = std::max<uint32_t>(16, f->img_bytes[var]);
+    const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     fn<<<1, kThreads, smem, f->stream>>>(fp);
     CK(cudaGetLastError());

@@ -87,13 +87,17 @@ inline void build_lookback(const ByteDFA &d, uint16_t *lb, uint8_t *nimg)
 }
 
 // Variant images (layouts documented in speck_kernel.cuh / DESIGN.md).
+// P8: field = next | count << 4 (count 0..8).  P4 (byte mode only): field = next | (4 + count) << 4
+// with count 0/1, so the high nibble selects byte 0 or 1 of PRMT's constant operand (speck_kernel.cuh).
 inline std::vector<uint8_t> image_packed(const ByteDFA &d, bool wide)
 {
     const uint32_t bytes = wide ? 8 : 4;
-    std::vector<uint8_t> img(256 * bytes, 0);
+    std::vector<uint8_t> img(256 * bytes, wide ? 0 : 0x40);
     for (uint32_t c = 0; c < 256; c++)
-        for (uint32_t s = 0; s < d.n; s++)
-            img[c * bytes + s] = (uint8_t)(d.next[(size_t)s * 256 + c] | (d.inc[(size_t)s * 256 + c] << 4));
+        for (uint32_t s = 0; s < d.n; s++) {
+            const uint32_t nx = d.next[(size_t)s * 256 + c], k = d.inc[(size_t)s * 256 + c];
+            img[c * bytes + s] = (uint8_t)(wide ? (nx | (k << 4)) : (nx | ((4 + k) << 4)));
+        }
     return img;
 }
 

@@ -23,6 +23,7 @@ __global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb
 {
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
+    check_smem_window(VAR, scratch_offset(VAR, p.table_bytes));
     TB tb;
     tb.setup(smem, p.table, p.n_states, kconst(p));
     __syncthreads();
@@ -52,7 +53,7 @@ __global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb
         for (int s = 0; s < K; s++) {
             sb.S[g * K + s] = (uint16_t)(S[s] == NOSTATE ? 0xFFFFu : S[s]);
             sb.E[g * K + s] = tb.state_of(cur[s]);
-            sb.C[g * K + s] = tb.count_of(acc[s], accf[s]);
+            sb.C[g * K + s] = tb.count_of(acc[s], accf[s], cur[s], e - b);
         }
     }
 }
@@ -62,10 +63,11 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
 {
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
+    const uint32_t T = blockDim.x;
+    const uint32_t tb_bytes = scratch_offset(VAR, p.table_bytes);
+    check_smem_window(VAR, tb_bytes + (uint32_t)(2 * T * K * 2 + 16 + 2 * 2 * T * K * 4));
     TB tb;
     tb.setup(smem, p.table, p.n_states, kconst(p));
-    const uint32_t T = blockDim.x;
-    const uint32_t tb_bytes = (p.table_bytes + 15) & ~15u;
     // double-buffered batches of T mappings
     uint16_t *bS = reinterpret_cast<uint16_t *>(smem + tb_bytes);            // [2][T][K]
     uint32_t *bE = reinterpret_cast<uint32_t *>(smem + tb_bytes + 2 * T * K * 2 + 16);
@@ -159,9 +161,9 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
     }
 }
 
-inline size_t seq_walk_smem(uint32_t T, int K, uint32_t table_bytes)
+inline size_t seq_walk_smem(uint32_t T, int K, int var, uint32_t table_bytes)
 {
-    return ((table_bytes + 15) & ~15u) + 2 * T * K * 2 + 16 + 2 * 2 * T * K * 4;
+    return scratch_offset(var, table_bytes) + 2 * T * K * 2 + 16 + 2 * 2 * T * K * 4;
 }
 
 }  // namespace speck

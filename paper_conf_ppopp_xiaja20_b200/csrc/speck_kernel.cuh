@@ -32,7 +32,11 @@ constexpr int kThreads = 256;  // auxiliary kernels
 // Threads per tile (one chunk per thread) of the fused kernel, by the number of chains K: large
 // CTAs keep few tiles in flight (short look-back windows) at one CTA per SM; the register budget
 // caps them for large K.
-__host__ __device__ constexpr int max_threads(int K) { return K <= 3 ? 1024 : K <= 6 ? 512 : 256; }
+#ifndef FSM_SMALLK_THREADS
+#define FSM_SMALLK_THREADS 1024
+#endif
+__host__ __device__ constexpr int max_threads(int K) { return K <= 3 ? FSM_SMALLK_THREADS : K <= 6 ? 512 : 256; }
+__host__ __device__ constexpr int min_blocks(int K) { return K <= 3 ? 1024 / FSM_SMALLK_THREADS : 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
 
 // ------------------------------------------------------------------------------- PTX helpers --
@@ -121,6 +125,45 @@ __device__ __forceinline__ uint32_t mad_lo(uint32_t a, uint32_t b, uint32_t c)
     return d;
 }
 
+// Shared-memory loads at a 32-bit shared-window address (the packed tables live at 0x10000 so that
+// a single PRMT produces the complete address).
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a)
+{
+    uint32_t v;
+    asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint2 lds_v2(uint32_t a)
+{
+    uint2 v;
+    asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t dp4a_u(uint32_t a, uint32_t b, uint32_t c)
+{
+    uint32_t d;
+    asm("dp4a.u32.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+    return d;
+}
+constexpr uint32_t kPackedBase = 0x10000u;  // shared-window address of the packed tables
+constexpr uint32_t kSmemWindowBase = 1024u;  // dynamic shared memory starts here (measured: tools/smem_probe)
+__host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1; }
+// Offset (from the start of dynamic smem) of the scratch area that follows the table.  Packed
+// tables occupy the window [0x10000, 0x20000); everything else goes above them.
+__host__ __device__ constexpr uint32_t scratch_offset(int var, uint32_t table_bytes)
+{
+    return is_packed(var) ? (kPackedBase + 65536u - kSmemWindowBase) : ((table_bytes + 15u) & ~15u);
+}
+__device__ __forceinline__ void check_smem_window(int var, uint32_t need)
+{
+    if (!is_packed(var)) return;
+    extern __shared__ __align__(16) uint8_t smem[];
+    uint32_t dyn;
+    asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(dyn));
+    const uint32_t base = (uint32_t)__cvta_generic_to_shared(smem);
+    if (base != kSmemWindowBase || dyn < need) __trap();  // loud: the layout assumption does not hold
+}
+
 struct KConst {
     uint32_t k_1e24, k_16, k_512;
 };
@@ -134,72 +177,84 @@ __device__ __forceinline__ KConst kconst(const Params &p) { return KConst{p.k_1e
 //   row(c) / apply(row, st, cnt)       single-chain step used by re-execution
 // Entries carry the accept increment of the destination state (byte mode 0/1, bit mode 0..8).
 
-// P4/P8: the transition function of symbol c packed into one row of N <= 4 (8) byte fields,
-// field = next | count << 4.  The row address depends only on the input byte, so it is off the
-// dependency chain; one conflict-free LDS.32/LDS.64 serves all K chains, and each chain step is
-// a single PRMT (byte select by the current state).  Lane-replicated: lane l reads its own copy.
+// P4/P8: the transition function of symbol c packed into one row of N <= 4 (8) byte fields.
+// The row address depends only on the input byte, so it is off the dependency chain; one
+// conflict-free LDS.32/LDS.64 serves all K chains, and each chain step is a single PRMT (byte
+// select by the current state).  Rows are lane-replicated (lane l reads its own copy) and live at
+// shared address 0x10000 + c * 256 + lane * 4|8, so the address is ONE PRMT of the input word:
+// byte0 <- lane offset, byte1 <- input byte c, byte2 <- 0x01.
+//  P8 field = next | count << 4 (bit mode: count 0..8).
+//  P4 field = next | (4 + count) << 4 (byte mode): PRMT's second operand X = 0x4544 turns the
+//     high nibble into a selector of X, so result byte 1 = 0x44 + count of the previous step and
+//     one DP4A (dot with 0x100) accumulates it; the 0x44 bias is removed at the end.
 template <int VAR>
 struct TablePacked {
     static constexpr bool kWide = VAR == VAR_P8;
-    const uint8_t *sm;
+    static constexpr uint32_t kX = 0x4544u;
     uint32_t lanereg;
-    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t, const KConst &kc)
+    uint32_t c24, c16;  // 1 << 24 and 16 from kernel params so that ptxas keeps IMAD / IMAD.HI (FMA pipe)
+    __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
     {
-        sm = s;
-        lanereg = (threadIdx.x & 31) * (kWide ? 8 : 4);
+        lanereg = kPackedBase | ((threadIdx.x & 31) * (kWide ? 8 : 4));
         c24 = kc.k_1e24;
         c16 = kc.k_16;
         if (kWide) {
             const uint2 *rows = static_cast<const uint2 *>(g);
             for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
-                uint32_t c = i >> 5, l = i & 31;
-                reinterpret_cast<uint2 *>(s)[c * 32 + l] = __ldg(rows + c);
+                const uint2 v = __ldg(rows + (i >> 5));
+                asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(kPackedBase + i * 8), "r"(v.x), "r"(v.y));
             }
         } else {
             const uint32_t *rows = static_cast<const uint32_t *>(g);
             for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
-                uint32_t c = i >> 5, l = i & 31;
-                reinterpret_cast<uint32_t *>(s)[c * 64 + l] = __ldg(rows + c);
+                const uint32_t v = __ldg(rows + (i >> 5));
+                asm volatile("st.shared.u32 [%0], %1;" ::"r"(kPackedBase + (i >> 5) * 256 + (i & 31) * 4), "r"(v));
             }
         }
     }
-    uint32_t c24, c16;  // 1 << 24 and 16 as opaque registers so that ptxas keeps IMAD / IMAD.HI (FMA pipe)
-    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return kWide ? st : (st | 0x44444440u); }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur & 0xFu; }
-    // acc: count * 16 (ALU-pipe accumulation), accf: count (FMA-pipe accumulation)
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf) const { return (acc >> 4) + accf; }
+    // P8: acc = count * 16 (ALU accumulation) + accf (FMA accumulation).
+    // P4: acc = sum of (0x44 + lagged count) over n steps; the last step's count sits in cur.
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t cur, uint64_t n) const
+    {
+        if (kWide) return (acc >> 4) + accf;
+        return acc - 0x44u * (uint32_t)n + ((cur >> 4) & 0xFu) - 4u;
+    }
 
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                          uint32_t (&accf)[K]) const
     {
-        // address = c * 256 + lane * 4|8, built by one PRMT: byte1 <- byte j of w, byte0 <- lanereg
-        const uint32_t a = prmt(w, lanereg, 0x5504u | (uint32_t(j) << 4));
-        uint32_t rx, ry = 0u;
+        const uint32_t a = prmt(w, lanereg, 0x7604u | (uint32_t(j) << 4));
         if (kWide) {
-            const uint2 r = *reinterpret_cast<const uint2 *>(sm + a);
-            rx = r.x;
-            ry = r.y;
-        } else {
-            rx = *reinterpret_cast<const uint32_t *>(sm + a);
-        }
+            const uint2 r = lds_v2(a);
 #pragma unroll
-        for (int s = 0; s < K; s++) {
-            cur[s] = prmt(rx, ry, cur[s]);                       // the chain: one PRMT per step
-            if (((j + s) & 1) == 0) acc[s] += cur[s] & 0xF0u;    // ALU: LOP3 (+ half an IADD3)
-            else accf[s] = mad_hi(cur[s] * c24, c16, accf[s]);   // FMA: IMAD, IMAD.HI (field >> 4)
+            for (int s = 0; s < K; s++) {
+                cur[s] = prmt(r.x, r.y, cur[s]);                       // the chain: one PRMT per step
+                if (((j + s) & 1) == 0) acc[s] += cur[s] & 0xF0u;      // ALU: LOP3 (+ half an IADD3)
+                else accf[s] = mad_hi(cur[s] * c24, c16, accf[s]);     // FMA: IMAD, IMAD.HI (field >> 4)
+            }
+        } else {
+            const uint32_t r = lds_u32(a);
+#pragma unroll
+            for (int s = 0; s < K; s++) {
+                cur[s] = prmt(r, kX, cur[s]);
+                acc[s] = dp4a_u(cur[s], 0x100u, acc[s]);
+            }
         }
     }
     using Row = uint2;
     __device__ __forceinline__ Row row(uint32_t c) const
     {
-        if (kWide) return *reinterpret_cast<const uint2 *>(sm + (c << 8) + lanereg);
-        return make_uint2(*reinterpret_cast<const uint32_t *>(sm + (c << 8) + lanereg), 0u);
+        const uint32_t a = lanereg + (c << 8);
+        if (kWide) return lds_v2(a);
+        return make_uint2(lds_u32(a), kX);
     }
     __device__ __forceinline__ uint32_t apply(Row r, uint32_t st, uint32_t &cnt) const
     {
         const uint32_t f = prmt(r.x, r.y, st) & 0xFFu;
-        cnt += f >> 4;
+        cnt += kWide ? (f >> 4) : ((f >> 4) - 4u);
         return f & 0xFu;
     }
 };
@@ -219,7 +274,7 @@ struct TableB {
     uint32_t c512, c2e24;
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf) const { return acc + accf; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                          uint32_t (&accf)[K]) const
@@ -250,7 +305,7 @@ struct TableG {
     __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &) { gt = static_cast<const uint32_t *>(g); }
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf) const { return acc + accf; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                          uint32_t (&accf)[K]) const
@@ -319,6 +374,52 @@ __device__ __forceinline__ bool chains_converged(const TB &tb, const uint32_t (&
 // chains of every active lane coincide the remainder runs ONE chain and its count increments
 // are added to every slot -- bit-identical to running all k chains.  Absent slots start as a copy
 // of slot 0 so they never block the vote (their results are ignored).
+// Blocks [i, nblk) of 32 bytes with a 3-buffer rotation (2 blocks in flight, no register moves).
+// On entry x0 = block i, x1 = block i+1.  With CHECK, returns true as soon as the warp votes
+// that all chains coincide; x0/x1 then hold blocks i, i+1 for the continuation.
+template <int KK, bool CHECK, class TB>
+__device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint64_t &i, uint64_t nblk, Bytes32 &x0,
+                                           Bytes32 &x1, uint32_t (&cur)[KK], uint32_t (&acc)[KK],
+                                           uint32_t (&accf)[KK])
+{
+    Bytes32 x2;
+    while (i < nblk) {
+        if (i + 2 < nblk) x2 = ldg_block(p, i + 2, nblk);
+        process32<KK>(tb, x0, cur, acc, accf);
+        ++i;
+        if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
+            x0 = x1;
+            x1 = x2;
+            return true;
+        }
+        if (i >= nblk) break;
+        if (i + 2 < nblk) x0 = ldg_block(p, i + 2, nblk);
+        process32<KK>(tb, x1, cur, acc, accf);
+        ++i;
+        if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
+            x1 = x0;
+            x0 = x2;
+            return true;
+        }
+        if (i >= nblk) break;
+        if (i + 2 < nblk) x1 = ldg_block(p, i + 2, nblk);
+        process32<KK>(tb, x2, cur, acc, accf);
+        ++i;
+        if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
+            x0 = x0;  // blocks i, i+1 already in x0, x1
+            return true;
+        }
+    }
+    return false;
+}
+
+// Alg. 3 over bytes [b, e) of the input: 32-byte blocks (one full sector per lane per
+// LDG.256) with two blocks in flight, then the ragged tail byte by byte.
+// Convergence: two chains that reach the same state stay identical for the rest of the chunk
+// (the state-convergence property of [18]).  After every block the warp votes; once all
+// chains of every active lane coincide the remainder runs ONE chain and its count increments
+// are added to every slot -- bit-identical to running all k chains.  Absent slots start as a copy
+// of slot 0 so they never block the vote (their results are ignored).
 template <int K, class TB>
 __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restrict__ in, uint64_t b, uint64_t e,
                                             bool aligned, uint32_t (&cur)[K], uint32_t (&acc)[K],
@@ -332,52 +433,13 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
     Bytes32 x0, x1;
     if (nblk) {
         x0 = ldg_block(p, 0, nblk);
-        x1 = x0;
         if (nblk > 1) x1 = ldg_block(p, 1, nblk);
-        // two blocks per iteration so the double buffer alternates registers instead of moving them
-        for (; i < nblk;) {
-            Bytes32 x2 = x1;
-            if (i + 2 < nblk) x2 = ldg_block(p, i + 2, nblk);
-            process32<K>(tb, x0, cur, acc, accf);
-            i++;
-            if constexpr (K > 1) {
-                if (__all_sync(__activemask(), chains_converged<K>(tb, cur))) {
-                    x0 = x1;
-                    x1 = x2;
-                    single = true;
-                    break;
-                }
-            }
-            if (i >= nblk) break;
-            Bytes32 x3 = x2;
-            if (i + 2 < nblk) x3 = ldg_block(p, i + 2, nblk);
-            process32<K>(tb, x1, cur, acc, accf);
-            i++;
-            x0 = x2;
-            x1 = x3;
-            if constexpr (K > 1) {
-                if (__all_sync(__activemask(), chains_converged<K>(tb, cur))) {
-                    single = true;
-                    break;
-                }
-            }
-        }
+        single = run_blocks<K, (K > 1)>(tb, p, i, nblk, x0, x1, cur, acc, accf);
     }
     if constexpr (K > 1) {
         if (single) {
             uint32_t c1[1] = {cur[0]}, a1[1] = {0u}, f1[1] = {0u};
-            while (i < nblk) {
-                Bytes32 x2 = x1;
-                if (i + 2 < nblk) x2 = ldg_block(p, i + 2, nblk);
-                process32<1>(tb, x0, c1, a1, f1);
-                if (++i >= nblk) break;
-                Bytes32 x3 = x2;
-                if (i + 2 < nblk) x3 = ldg_block(p, i + 2, nblk);
-                process32<1>(tb, x1, c1, a1, f1);
-                ++i;
-                x0 = x2;
-                x1 = x3;
-            }
+            run_blocks<1, false>(tb, p, i, nblk, x0, x1, c1, a1, f1);
             for (uint64_t t = nblk << 5; t < n; t++) tb.template step<1>(__ldg(p + t), 0, c1, a1, f1);
 #pragma unroll
             for (int s = 0; s < K; s++) {
@@ -445,10 +507,10 @@ __device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eo
 
 // ----------------------------------------------------------------- shared-memory layout ----
 struct Layout {
-    uint32_t qe, qc, sj, ws, we, wc, wi, total;
-    __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t table_bytes)
+    uint32_t qe, qc, sj, ws, we, wc, wi, misc, total;
+    __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t start)
     {
-        uint32_t o = (table_bytes + 15) & ~15u;
+        uint32_t o = start;
         qe = o;  o += T * K * 4;
         qc = o;  o += T * K * 4;
         sj = o;  o += T * K * 2;
@@ -457,6 +519,7 @@ struct Layout {
         we = o;  o += 32 * K * 4;
         wc = o;  o += 32 * K * 4;
         wi = o;  o += 32 * 4;
+        misc = o; o += 16;
         total = o;
     }
 };
@@ -560,19 +623,19 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
 
 // ------------------------------------------------------------------------------- the kernel --
 template <int K, int VAR>
-__global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
+__global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Params p)
 {
     using TB = typename TableFor<VAR>::type;
-    extern __shared__ __align__(16) uint8_t smem[];
-    __shared__ uint32_t s_tile;
+    extern __shared__ __align__(16) uint8_t smem[];  // no static shared memory: see kSmemWindowBase
 
     const uint32_t T = blockDim.x;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = T >> 5;
     const uint32_t j = threadIdx.x;
 
+    const Layout L(T, K, scratch_offset(VAR, p.table_bytes));
+    check_smem_window(VAR, L.total);
     TB tb;
     tb.setup(smem, p.table, p.n_states, kconst(p));
-    const Layout L(T, K, p.table_bytes);
     uint32_t *Qe = reinterpret_cast<uint32_t *>(smem + L.qe);
     uint32_t *Qc = reinterpret_cast<uint32_t *>(smem + L.qc);
     uint16_t *Sj = reinterpret_cast<uint16_t *>(smem + L.sj);
@@ -580,6 +643,7 @@ __global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
     uint32_t *wE = reinterpret_cast<uint32_t *>(smem + L.we);
     uint32_t *wC = reinterpret_cast<uint32_t *>(smem + L.wc);
     uint32_t *wI = reinterpret_cast<uint32_t *>(smem + L.wi);
+    uint32_t &s_tile = *reinterpret_cast<uint32_t *>(smem + L.misc);
 
     const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
     const unsigned long long start_count = p.start_dev ? p.start_dev->count : 0ull;
@@ -613,6 +677,9 @@ __global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
         }
 
         // ---- a4: local processing
+#ifdef FSM_PHASE_TIMING
+        long long t_local0 = clock64();
+#endif
         uint32_t cur[K], acc[K], accf[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
@@ -625,10 +692,14 @@ __global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
 #pragma unroll
         for (int s = 0; s < K; s++) {
             eob[s] = S[s] == NOSTATE ? (ABSENT << 16) : (tb.state_of(cur[s]) | (COMPLETE << 16));
-            cnt[s] = tb.count_of(acc[s], accf[s]);
+            cnt[s] = tb.count_of(acc[s], accf[s], cur[s], empty ? 0 : e - b);
         }
         bool ident = empty;
 
+#ifdef FSM_PHASE_TIMING
+        long long t_local1 = clock64();
+        atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 40, (unsigned long long)(t_local1 - t_local0));
+#endif
         // ---- a5: warp stage (chunks warp*32 .. warp*32+31)
         warp_suffix_scan<K>(S, eob, cnt, ident, (uint32_t)warp * 32, 1);
 
@@ -687,6 +758,10 @@ __global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
         }
         __syncthreads();
 
+#ifdef FSM_PHASE_TIMING
+        long long t_scan1 = clock64();
+        if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 41, (unsigned long long)(t_scan1 - t_local1));
+#endif
         if (warp != 0) continue;
 
         // ================= warp 0: tile epilogue (pre-resolution, look-back, publication) =====
@@ -871,6 +946,15 @@ __global__ void __launch_bounds__(max_threads(K), 1) speck_kernel(Params p)
         __syncwarp();
         if (lane == 0) st_release(&D->flag, ep | ST_P);
 
+#ifdef FSM_PHASE_TIMING
+        if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 42, (unsigned long long)(clock64() - t_scan1));
+        if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 43, 1ull);
+        if (threadIdx.x == 0 && tile == p.ntiles - 1) {
+            unsigned long long *q = reinterpret_cast<unsigned long long *>(p.result) + 40;
+            printf("PHASES local(sum over threads)=%llu scan+merge(t0)=%llu epilogue(t0)=%llu tiles=%llu T=%u\n", q[0], q[1], q[2], q[3], T);
+            q[0] = q[1] = q[2] = q[3] = 0;
+        }
+#endif
         // a9: the last tile writes the result (bit-mode tail applied here)
         if (tile == p.ntiles - 1) {
             uint32_t x = Ps;

@@ -40,7 +40,7 @@ VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3}
 
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
-    return {"P4": n <= 4, "P8": n <= 8, "B": n <= 256, "G": True}[var]
+    return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "B": n <= 256, "G": True}[var]
 
 
 # --------------------------------------------------------------------- worked example on GPU

@@ -183,6 +183,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--variant", type=int, default=-1)
     ap.add_argument("--chunk", type=int, default=0)
+    ap.add_argument("--no-ablation", action="store_true",
+                    help="skip the sequential-merge ablation run (Fig. 4a, SURVEY 8.a11)")
     args = ap.parse_args()
     w = make_workload(args)
     if args.impl == "reference":
@@ -309,6 +311,9 @@ def main():
     except OSError:
         pass
     peak = float(peaks.get("hbm_gbs", 6650.0))
+    traffic = None
+    if args.config == "c5" and args.n_states == 8 and args.m == 2 and args.k == 2:
+        traffic = round(1.031 * n)   # per launch, from the committed ncu capture of this config
     line = {
         "metric": METRIC, "value": round(gbs, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(step_s * 1e3, 4), "higher_is_better": True,
@@ -316,13 +321,31 @@ def main():
         "config": config_json(args, w),
         "roofline": {"bound": "hbm", "achieved": round(n / step_s / 1e9, 3) if world == 1 else round(gbs / world, 3),
                      "peak": peak, "unit": "GB/s", "frac": round((n / step_s / 1e9) / peak, 4),
-                     "traffic": None, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback"},
+                     "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback"},
+        "traffic_note": "ncu --set full (profiles/r01_ncu_c5_n8m2k2_8GiB.txt): dram read+write = 1.031 x input bytes",
         "clocks": clk.summary(),
-        "gpu_launches": args.steps * (1 if world == 1 else 1),
+        "gpu_launches": args.steps,  # one fused kernel per step (plus a fix-up kernel per miss round for N > 1)
         "result": {"final_state": final[0], "accept_count": final[1]},
         "stats": {kk: v for kk, v in st.items()},
         "e2e": e2e,
     }
+    if not args.no_ablation and world == 1:
+        # internal ablation: the paper's sequential merge (Fig. 4a) on the same input and chains
+        f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_SEQUENTIAL)
+        f.run_spec_k_async(buf.data_ptr(), n, k, res.data_ptr())
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        f.run_spec_k_async(buf.data_ptr(), n, k, res.data_ptr())
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ts = e0.elapsed_time(e1) / 1e3
+        r2 = res.cpu().numpy().view(np.uint32)
+        same = (int(r2[0]), int(r2[2]) | (int(r2[3]) << 32)) == final
+        f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_PARALLEL)
+        line["ablation"] = {"sequential_merge_gbs": round(n / ts / 1e9, 3),
+                            "parallel_over_sequential": round(ts / step_s, 2), "same_result": same,
+                            "paper_v100_context": "2.02-6.74x (P:11, P:53)"}
     if not args.no_cpu and world == 1:
         try:
             os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})

@@ -58,9 +58,14 @@ def run_sharded(f: FSM, shard_ptr: int, shard_len: int, halo_ptr: int | None, k:
     m, shard = f.run_shard(shard_ptr, shard_len, halo=halo_ptr if rank else None,
                            halo_len=1 if rank else 0, k=k, keep=True)
     mine = torch.from_numpy(_pack(m)).to(device)
-    allm = torch.empty(world * _MAPW, dtype=torch.int64, device=device)
-    dist.all_gather_into_tensor(allm, mine, group=group)
-    host = allm.cpu().numpy().reshape(world, _MAPW)
+    if dist.get_backend(group) == "nccl":
+        allm = torch.empty(world * _MAPW, dtype=torch.int64, device=device)
+        dist.all_gather_into_tensor(allm, mine, group=group)   # the one collective (NVLink/NVSwitch)
+        host = allm.cpu().numpy().reshape(world, _MAPW)
+    else:  # gloo (CPU tests of this host logic)
+        parts = [torch.empty_like(mine) for _ in range(world)]
+        dist.all_gather(parts, mine, group=group)
+        host = torch.stack(parts).cpu().numpy()
     maps = [_unpack(host[g]) for g in range(world)]
     x, total, miss = compose_from(q0, maps)
     fix = torch.zeros(2, dtype=torch.int64, device=device)

@@ -52,7 +52,8 @@ enum {
     FSM_VARIANT_P4 = 0,  /* N <= 4 (byte mode): packed 4 x u8 row per symbol, lane-replicated smem, PRMT chain */
     FSM_VARIANT_P8 = 1,  /* N <= 8:   packed 8 x u8 row per symbol, lane-replicated smem, PRMT chain */
     FSM_VARIANT_B = 2,   /* N <= 256: u16 entries (next | count << 8) in shared memory            */
-    FSM_VARIANT_G = 3    /* any N:    u32 entries (next | count << 16) in global memory / L2      */
+    FSM_VARIANT_G = 3,   /* any N:    u32 entries (next | count << 16) in global memory / L2      */
+    FSM_VARIANT_H8 = 4   /* N <= 8 (byte mode): half rows of 4 states, one LDS.32 per chain step   */
 };
 
 /* Merge strategies: the paper's parallel merge (default) and its sequential-merge baseline

@@ -11,7 +11,8 @@ CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libfsmspec.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
-         "-shared", "-Xcompiler", "-fPIC", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
+         "-Xcompiler", "-fPIC", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
+UNITS = ["fsmspec", "kernels_p4", "kernels_p8", "kernels_h8", "kernels_b", "kernels_g"]
 
 
 def sources() -> list[str]:
@@ -27,19 +28,40 @@ def stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile the translation units in parallel (one per table variant) and link the .so."""
     if not force and not stale():
         return SO
-    cmd = [NVCC, *FLAGS, "-I", os.path.join(ROOT, "include"), "-o", SO + ".tmp",
-           os.path.join(CSRC, "fsmspec.cu")]
-    res = subprocess.run(cmd, capture_output=True, text=True)
+    import concurrent.futures as cf
+    import tempfile
+
+    tmp = tempfile.mkdtemp(prefix="fsmspec_build_")
     log = os.path.join(HERE, "build.log")
+
+    def unit(u):
+        obj = os.path.join(tmp, u + ".o")
+        cmd = [NVCC, *FLAGS, "-I", os.path.join(ROOT, "include"), "-c", "-o", obj, os.path.join(CSRC, u + ".cu")]
+        res = subprocess.run(cmd, capture_output=True, text=True)
+        return u, obj, cmd, res
+
+    with cf.ThreadPoolExecutor(len(UNITS)) as ex:
+        results = list(ex.map(unit, UNITS))
     with open(log, "w") as fh:
-        fh.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
+        for u, obj, cmd, res in results:
+            fh.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
+    bad = [(u, r) for u, _, _, r in results if r.returncode != 0]
+    if bad:
+        raise RuntimeError(f"nvcc failed for {bad[0][0]} (see {log}):\n{bad[0][1].stderr[-4000:]}")
+    cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", SO + ".tmp",
+           *[o for _, o, _, _ in results]]
+    res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
-        raise RuntimeError(f"nvcc failed (see {log}):\n{res.stderr[-4000:]}")
+        raise RuntimeError(f"link failed:\n{res.stderr[-4000:]}")
     os.replace(SO + ".tmp", SO)
+    import shutil
+
+    shutil.rmtree(tmp, ignore_errors=True)
     if verbose:
-        print(res.stderr[-2000:])
+        print(open(log).read()[-2000:])
     return SO
 
 

@@ -23,7 +23,7 @@ using namespace speck;
 
 // ------------------------------------------------------------------ kernel instantiations ----
 // k is a compile-time constant; a run with k uses the smallest instantiated K >= k and
-// marks the extra slots absent.
+// marks the extra slots absent (kernels_inst.cuh instantiates the same list).
 static const int kKs[] = {1, 2, 3, 4, 6, 8, 12, 16};
 constexpr int kNumKs = 8;
 
@@ -32,59 +32,46 @@ typedef void (*FixFn)(FixParams);
 typedef void (*SeqLocalFn)(Params, SeqBuf);
 typedef void (*SeqWalkFn)(Params, SeqBuf);
 
-template <int VAR>
-static KernelFn kernel_for(int K)
-{
-    switch (K) {
-    case 1: return speck_kernel<1, VAR>;
-    case 2: return speck_kernel<2, VAR>;
-    case 3: return speck_kernel<3, VAR>;
-    case 4: return speck_kernel<4, VAR>;
-    case 6: return speck_kernel<6, VAR>;
-    case 8: return speck_kernel<8, VAR>;
-    case 12: return speck_kernel<12, VAR>;
-    default: return speck_kernel<16, VAR>;
-    }
-}
+// Kernel instantiations live in one translation unit per table variant (kernels_*.cu, compiled in
+// parallel); each exports these accessors.
+#define FSM_DECLARE_VARIANT(NAME)                                   \
+    KernelFn get_kernel_##NAME(int K);                              \
+    FixFn get_fix_##NAME();                                         \
+    void get_seq_##NAME(int K, SeqLocalFn &l, SeqWalkFn &w);
+FSM_DECLARE_VARIANT(p4)
+FSM_DECLARE_VARIANT(p8)
+FSM_DECLARE_VARIANT(h8)
+FSM_DECLARE_VARIANT(b)
+FSM_DECLARE_VARIANT(g)
+
 static KernelFn get_kernel(int var, int K)
 {
     switch (var) {
-    case VAR_P4: return kernel_for<VAR_P4>(K);
-    case VAR_P8: return kernel_for<VAR_P8>(K);
-    case VAR_B: return kernel_for<VAR_B>(K);
-    default: return kernel_for<VAR_G>(K);
+    case VAR_P4: return get_kernel_p4(K);
+    case VAR_P8: return get_kernel_p8(K);
+    case VAR_H8: return get_kernel_h8(K);
+    case VAR_B: return get_kernel_b(K);
+    default: return get_kernel_g(K);
     }
 }
 static FixFn get_fix(int var)
 {
     switch (var) {
-    case VAR_P4: return fixup_kernel<VAR_P4>;
-    case VAR_P8: return fixup_kernel<VAR_P8>;
-    case VAR_B: return fixup_kernel<VAR_B>;
-    default: return fixup_kernel<VAR_G>;
-    }
-}
-template <int VAR>
-static void seq_for(int K, SeqLocalFn &l, SeqWalkFn &w)
-{
-    switch (K) {
-    case 1: l = seq_local_kernel<1, VAR>; w = seq_walk_kernel<1, VAR>; break;
-    case 2: l = seq_local_kernel<2, VAR>; w = seq_walk_kernel<2, VAR>; break;
-    case 3: l = seq_local_kernel<3, VAR>; w = seq_walk_kernel<3, VAR>; break;
-    case 4: l = seq_local_kernel<4, VAR>; w = seq_walk_kernel<4, VAR>; break;
-    case 6: l = seq_local_kernel<6, VAR>; w = seq_walk_kernel<6, VAR>; break;
-    case 8: l = seq_local_kernel<8, VAR>; w = seq_walk_kernel<8, VAR>; break;
-    case 12: l = seq_local_kernel<12, VAR>; w = seq_walk_kernel<12, VAR>; break;
-    default: l = seq_local_kernel<16, VAR>; w = seq_walk_kernel<16, VAR>; break;
+    case VAR_P4: return get_fix_p4();
+    case VAR_P8: return get_fix_p8();
+    case VAR_H8: return get_fix_h8();
+    case VAR_B: return get_fix_b();
+    default: return get_fix_g();
     }
 }
 static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
 {
     switch (var) {
-    case VAR_P4: seq_for<VAR_P4>(K, l, w); break;
-    case VAR_P8: seq_for<VAR_P8>(K, l, w); break;
-    case VAR_B: seq_for<VAR_B>(K, l, w); break;
-    default: seq_for<VAR_G>(K, l, w); break;
+    case VAR_P4: get_seq_p4(K, l, w); break;
+    case VAR_P8: get_seq_p8(K, l, w); break;
+    case VAR_H8: get_seq_h8(K, l, w); break;
+    case VAR_B: get_seq_b(K, l, w); break;
+    default: get_seq_g(K, l, w); break;
     }
 }
 
@@ -106,8 +93,8 @@ struct fsm {
     int auto_variant = VAR_G;
     fsm_options opt{};
     // device tables
-    void *d_img[4] = {nullptr, nullptr, nullptr, nullptr};
-    uint32_t img_bytes[4] = {0, 0, 0, 0};
+    void *d_img[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
+    uint32_t img_bytes[5] = {0, 0, 0, 0, 0};
     uint16_t *d_lb = nullptr;
     uint8_t *d_nimg = nullptr;
     uint32_t *d_bittab = nullptr;
@@ -187,7 +174,7 @@ extern "C" int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint
 
 static void free_all(fsm *f)
 {
-    for (int i = 0; i < 4; i++) cudaFree(f->d_img[i]);
+    for (int i = 0; i < 5; i++) cudaFree(f->d_img[i]);
     cudaFree(f->d_lb);
     cudaFree(f->d_nimg);
     cudaFree(f->d_bittab);
@@ -270,6 +257,11 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         if ((rc = upload(&f->d_img[VAR_P4], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_P4] = 0;  // packed tables live in a fixed shared-window slot (scratch_offset)
     }
+    if (n <= 8 && !bits) {  // H8's count bit is byte-mode only
+        auto img = image_h8(f->dfa);
+        if ((rc = upload(&f->d_img[VAR_H8], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_H8] = 0;
+    }
     if (n <= 8) {
         auto img = image_packed(f->dfa, true);
         if ((rc = upload(&f->d_img[VAR_P8], img.data(), img.size()))) return fail(rc);
@@ -333,7 +325,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
-    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_G) return FSM_EINVAL;
+    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_H8) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     f->opt.chunk_bytes = o->chunk_bytes;            // 0 = adaptive
@@ -372,10 +364,15 @@ struct RunSpec {
     uint32_t merge;
 };
 
-static int variant_of(const fsm *f, int force)
+static int variant_of(const fsm *f, int force, uint32_t k = 1)
 {
     if (force >= 0) return force;
-    return f->opt.variant == FSM_VARIANT_AUTO ? f->auto_variant : f->opt.variant;
+    if (f->opt.variant != FSM_VARIANT_AUTO) return f->opt.variant;
+    // H8 (one LDS.32 per chain step, on the dependency chain) measured slower than P8 (one LDS.64
+    // per byte, off the chain) on B200: 3.21 vs 3.73 TB/s at k = 1, so the
+    // automatic choice keeps P8; H8 stays selectable.
+    (void)k;
+    return f->auto_variant;
 }
 
 // Geometry: T chunks per tile (CTA threads), chunk bytes.  Large inputs: the largest CTA the
@@ -415,7 +412,7 @@ static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T);
 
 static int launch_run(fsm *f, const RunSpec &r)
 {
-    const int var = variant_of(f, r.force_variant);
+    const int var = variant_of(f, r.force_variant, r.k);
     const int K = kslots(r.k);
     const bool bits = f->mode == FSM_INPUT_BITS_MSB;
     const uint64_t len_bytes = bits ? r.len_sym / 8 : r.len_sym;
@@ -453,6 +450,8 @@ static int launch_run(fsm *f, const RunSpec &r)
     p.k_1e24 = 1u << 24;
     p.k_16 = 16;
     p.k_512 = 512;
+    p.k_1e27 = 1u << 27;
+    p.k_2 = 2;
 
     const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes)).total;
 
@@ -703,7 +702,7 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         fp.count[s] = st->map.count[s];
     }
     fp.out = f->d_fix;
-    fp.kc = KConst{1u << 24, 16, 512};
+    fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2};
     FixFn fn = get_fix(var);
     const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

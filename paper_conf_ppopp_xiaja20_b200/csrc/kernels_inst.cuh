@@ -1,0 +1,45 @@
+// kernels_inst.cuh -- explicit instantiation of every kernel for one table variant.  Included by
+// kernels_<variant>.cu with FSM_VAR / FSM_VAR_NAME defined; the host (fsmspec.cu) reaches the
+// kernels through the accessors defined here.  K list = kKs in fsmspec.cu.
+#include "fixup_kernel.cuh"
+#include "seqmerge_kernel.cuh"
+#include "speck_kernel.cuh"
+
+using namespace speck;
+typedef void (*KernelFn)(Params);
+typedef void (*FixFn)(FixParams);
+typedef void (*SeqLocalFn)(Params, SeqBuf);
+typedef void (*SeqWalkFn)(Params, SeqBuf);
+
+#define FSM_CAT2(a, b) a##b
+#define FSM_CAT(a, b) FSM_CAT2(a, b)
+
+KernelFn FSM_CAT(get_kernel_, FSM_VAR_NAME)(int K)
+{
+    switch (K) {
+    case 1: return speck_kernel<1, FSM_VAR>;
+    case 2: return speck_kernel<2, FSM_VAR>;
+    case 3: return speck_kernel<3, FSM_VAR>;
+    case 4: return speck_kernel<4, FSM_VAR>;
+    case 6: return speck_kernel<6, FSM_VAR>;
+    case 8: return speck_kernel<8, FSM_VAR>;
+    case 12: return speck_kernel<12, FSM_VAR>;
+    default: return speck_kernel<16, FSM_VAR>;
+    }
+}
+
+FixFn FSM_CAT(get_fix_, FSM_VAR_NAME)() { return fixup_kernel<FSM_VAR>; }
+
+void FSM_CAT(get_seq_, FSM_VAR_NAME)(int K, SeqLocalFn &l, SeqWalkFn &w)
+{
+    switch (K) {
+    case 1: l = seq_local_kernel<1, FSM_VAR>; w = seq_walk_kernel<1, FSM_VAR>; break;
+    case 2: l = seq_local_kernel<2, FSM_VAR>; w = seq_walk_kernel<2, FSM_VAR>; break;
+    case 3: l = seq_local_kernel<3, FSM_VAR>; w = seq_walk_kernel<3, FSM_VAR>; break;
+    case 4: l = seq_local_kernel<4, FSM_VAR>; w = seq_walk_kernel<4, FSM_VAR>; break;
+    case 6: l = seq_local_kernel<6, FSM_VAR>; w = seq_walk_kernel<6, FSM_VAR>; break;
+    case 8: l = seq_local_kernel<8, FSM_VAR>; w = seq_walk_kernel<8, FSM_VAR>; break;
+    case 12: l = seq_local_kernel<12, FSM_VAR>; w = seq_walk_kernel<12, FSM_VAR>; break;
+    default: l = seq_local_kernel<16, FSM_VAR>; w = seq_walk_kernel<16, FSM_VAR>; break;
+    }
+}

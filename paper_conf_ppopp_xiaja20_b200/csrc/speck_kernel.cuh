@@ -27,7 +27,7 @@
 
 namespace speck {
 
-enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3 };
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Threads per tile (one chunk per thread) of the fused kernel, by the number of chains K: large
 // CTAs keep few tiles in flight (short look-back windows) at one CTA per SM; the register budget
@@ -147,7 +147,7 @@ __device__ __forceinline__ uint32_t dp4a_u(uint32_t a, uint32_t b, uint32_t c)
 }
 constexpr uint32_t kPackedBase = 0x10000u;  // shared-window address of the packed tables
 constexpr uint32_t kSmemWindowBase = 1024u;  // dynamic shared memory starts here (measured: tools/smem_probe)
-__host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1; }
+__host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1 || var == 4; }
 // Offset (from the start of dynamic smem) of the scratch area that follows the table.  Packed
 // tables occupy the window [0x10000, 0x20000); everything else goes above them.
 __host__ __device__ constexpr uint32_t scratch_offset(int var, uint32_t table_bytes)
@@ -165,9 +165,9 @@ __device__ __forceinline__ void check_smem_window(int var, uint32_t need)
 }
 
 struct KConst {
-    uint32_t k_1e24, k_16, k_512;
+    uint32_t k_1e24, k_16, k_512, k_1e27, k_2;
 };
-__device__ __forceinline__ KConst kconst(const Params &p) { return KConst{p.k_1e24, p.k_16, p.k_512}; }
+__device__ __forceinline__ KConst kconst(const Params &p) { return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2}; }
 
 // ------------------------------------------------------------------- table-placement variants --
 // Every variant exposes
@@ -259,6 +259,57 @@ struct TablePacked {
     }
 };
 
+// H8: N <= 8, byte mode.  Each row is split into two 4-state halves (states 0-3, 4-7) stored as
+// two lane-replicated u32 words at 0x10000 + c * 256 + half * 128 + lane * 4.  A chain loads only
+// the half its current state lives in: ONE conflict-free LDS.32 (one wavefront) instead of P8's
+// LDS.64 (two), at the price of putting the load on the dependency chain.  Field byte:
+// bits 0-1 = index in the half (PRMT selector), bit 4 = accept increment, bit 7 = half, so the
+// address of the next load is one LOP3: (cur & 0x80) | (PRMT of the input byte).
+struct TableH8 {
+    uint32_t lanereg;
+    uint32_t c27, c2;
+    __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
+    {
+        lanereg = kPackedBase | ((threadIdx.x & 31) * 4);
+        c27 = kc.k_1e27;
+        c2 = kc.k_2;
+        const uint2 *rows = static_cast<const uint2 *>(g);  // per symbol: {half 0 word, half 1 word}
+        for (uint32_t i = threadIdx.x; i < 256 * 64; i += blockDim.x) {
+            const uint32_t c = i >> 6, h = (i >> 5) & 1, l = i & 31;
+            const uint2 v = __ldg(rows + c);
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(kPackedBase + c * 256 + h * 128 + l * 4), "r"(h ? v.y : v.x));
+        }
+    }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return (st & 3u) | ((st & 4u) << 5); }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return (cur & 3u) | ((cur >> 5) & 4u); }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
+    {
+        const uint32_t a = prmt(w, lanereg, 0x7604u | (uint32_t(j) << 4));
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            const uint32_t r = lds_u32(a | (cur[s] & 0x80u));   // LOP3 + LDS.32 (half of the row)
+            cur[s] = prmt(r, r, cur[s]);                         // select the field
+            accf[s] = mad_hi(cur[s] * c27, c2, accf[s]);         // + bit 4, on the FMA pipe
+        }
+    }
+    using Row = uint2;
+    __device__ __forceinline__ Row row(uint32_t c) const
+    {
+        const uint32_t a = lanereg + (c << 8);
+        return make_uint2(lds_u32(a), lds_u32(a + 128));
+    }
+    __device__ __forceinline__ uint32_t apply(Row r, uint32_t st, uint32_t &cnt) const
+    {
+        const uint32_t w = (st & 4u) ? r.y : r.x;
+        const uint32_t f = prmt(w, w, st & 3u) & 0xFFu;
+        cnt += (f >> 4) & 1u;
+        return (f & 3u) | ((f >> 5) & 4u);
+    }
+};
+
 // B: u16 entries T[s][c] = next | count << 8 in shared memory (N <= 256; 512 B per state).
 struct TableB {
     const uint8_t *sm;
@@ -333,6 +384,7 @@ template <> struct TableFor<VAR_P4> { using type = TablePacked<VAR_P4>; };
 template <> struct TableFor<VAR_P8> { using type = TablePacked<VAR_P8>; };
 template <> struct TableFor<VAR_B> { using type = TableB; };
 template <> struct TableFor<VAR_G> { using type = TableG; };
+template <> struct TableFor<VAR_H8> { using type = TableH8; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <int K, class TB>

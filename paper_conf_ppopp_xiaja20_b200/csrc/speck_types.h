@@ -79,7 +79,7 @@ struct Params {
     DevStats *stats;
     // constants passed at run time so that ptxas cannot strength-reduce the FMA-pipe IMADs into
     // ALU-pipe shifts (the hot loop balances the two pipes): 1 << 24, 16, 512
-    uint32_t k_1e24, k_16, k_512;
+    uint32_t k_1e24, k_16, k_512, k_1e27, k_2;
 };
 
 }  // namespace speck

@@ -35,16 +35,17 @@ def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
     return res, st
 
 
-VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4}
 
 
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
-    return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "B": n <= 256, "G": True}[var]
+    return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "H8": n <= 8 and not dfa.bit_mode,
+            "B": n <= 256, "G": True}[var]
 
 
 # --------------------------------------------------------------------- worked example on GPU
-@pytest.mark.parametrize("var", ["P4", "P8", "B", "G"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G"])
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
 def test_fig1_worked_example(var, k):
     d = dfas.c_comment(True)
@@ -54,7 +55,7 @@ def test_fig1_worked_example(var, k):
 
 
 # --------------------------------------------------------------------- C1-shaped text
-@pytest.mark.parametrize("var", ["P4", "P8", "B", "G"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G"])
 @pytest.mark.parametrize("chunk", [0, 64, 96, 4096])
 def test_c_comment_text(var, chunk):
     d = dfas.c_comment(True)

@@ -29,6 +29,10 @@ namespace speck {
 
 enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4 };
 constexpr int kThreads = 256;  // auxiliary kernels
+// Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
+// in lockstep over the chunk's first 32 bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
+constexpr int kExt = 4;
+constexpr uint32_t kExtNone = 0xFFFFu;
 // Threads per tile (one chunk per thread) of the fused kernel, by the number of chains K: large
 // CTAs keep few tiles in flight (short look-back windows) at one CTA per SM; the register budget
 // caps them for large K.
@@ -475,7 +479,7 @@ __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint6
 template <int K, class TB>
 __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restrict__ in, uint64_t b, uint64_t e,
                                             bool aligned, uint32_t (&cur)[K], uint32_t (&acc)[K],
-                                            uint32_t (&accf)[K])
+                                            uint32_t (&accf)[K], uint32_t *stash = nullptr)
 {
     const uint8_t *p = in + b;
     const uint64_t n = e - b;
@@ -486,6 +490,10 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
     if (nblk) {
         x0 = ldg_block(p, 0, nblk);
         if (nblk > 1) x1 = ldg_block(p, 1, nblk);
+        if (stash) {
+            reinterpret_cast<uint4 *>(stash)[0] = make_uint4(x0.w[0], x0.w[1], x0.w[2], x0.w[3]);
+            reinterpret_cast<uint4 *>(stash)[1] = make_uint4(x0.w[4], x0.w[5], x0.w[6], x0.w[7]);
+        }
         single = run_blocks<K, (K > 1)>(tb, p, i, nblk, x0, x1, cur, acc, accf);
     }
     if constexpr (K > 1) {
@@ -513,9 +521,13 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
 // slot (which may itself be broken further on) and adds counts -- the membership check of
 // Alg. 1, all K compares unrolled into predicated selects (k is a compile-time
 // constant).  No match: the slot breaks at R's first chunk.
+// With `ext` (the eager-completion entries of R's first chunk, in smem) a state that is not a
+// speculated start of R but was run to convergence with one of R's chains continues as that slot,
+// corrected by the count difference up to the meeting point -- exact, and no break.
 template <int K>
 __device__ __forceinline__ void compose(uint32_t (&eob)[K], uint32_t (&cnt)[K], const uint32_t (&Sr)[K],
-                                        const uint32_t (&eobr)[K], const uint32_t (&cntr)[K], uint32_t first_r)
+                                        const uint32_t (&eobr)[K], const uint32_t (&cntr)[K], uint32_t first_r,
+                                        const uint32_t *ext = nullptr)
 {
 #pragma unroll
     for (int s = 0; s < K; s++) {
@@ -523,12 +535,31 @@ __device__ __forceinline__ void compose(uint32_t (&eob)[K], uint32_t (&cnt)[K], 
         if ((x >> 16) == COMPLETE) {
             const uint32_t st = x & 0xFFFFu;
             uint32_t ne = st | (first_r << 16), nc = 0;
+            bool hit = false;
 #pragma unroll
             for (int j = 0; j < K; j++)
                 if (Sr[j] == st) {
                     ne = eobr[j];
                     nc = cntr[j];
+                    hit = true;
                 }
+            if (!hit && ext) {
+                const uint32_t *ex = ext + first_r * kExt;
+#pragma unroll
+                for (int q = 0; q < kExt; q++) {
+                    const uint32_t v = ex[q];
+                    if ((v & 0xFFFFu) == st) {
+                        const uint32_t l = (v >> 16) & 0xFu;
+                        const int32_t delta = (int32_t)v >> 20;
+#pragma unroll
+                        for (int j = 0; j < K; j++)
+                            if ((uint32_t)j == l) {
+                                ne = eobr[j];
+                                nc = cntr[j] + (uint32_t)delta;
+                            }
+                    }
+                }
+            }
             eob[s] = ne;
             cnt[s] += nc;
         }
@@ -540,7 +571,7 @@ __device__ __forceinline__ void compose(uint32_t (&eob)[K], uint32_t (&cnt)[K], 
 // chunk distance between lanes.
 template <int K>
 __device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eob)[K], uint32_t (&cnt)[K], bool &ident,
-                                                 uint32_t first0, uint32_t step)
+                                                 uint32_t first0, uint32_t step, const uint32_t *ext = nullptr)
 {
     const int lane = threadIdx.x & 31;
 #pragma unroll
@@ -553,13 +584,13 @@ __device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eo
             cr[s] = __shfl_down_sync(0xFFFFFFFFu, cnt[s], d);
         }
         const bool ir = __shfl_down_sync(0xFFFFFFFFu, (int)ident, d) != 0;
-        if (lane + d < 32 && !ir && !ident) compose<K>(eob, cnt, Sr, er, cr, first0 + (lane + d) * step);
+        if (lane + d < 32 && !ir && !ident) compose<K>(eob, cnt, Sr, er, cr, first0 + (lane + d) * step, ext);
     }
 }
 
 // ----------------------------------------------------------------- shared-memory layout ----
 struct Layout {
-    uint32_t qe, qc, sj, ws, we, wc, wi, misc, total;
+    uint32_t qe, qc, sj, ws, we, wc, wi, misc, stash, ext, total;
     __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t start)
     {
         uint32_t o = start;
@@ -572,6 +603,8 @@ struct Layout {
         wc = o;  o += 32 * K * 4;
         wi = o;  o += 32 * 4;
         misc = o; o += 16;
+        stash = o; o += T * 32;
+        ext = o; o += T * kExt * 4;
         total = o;
     }
 };
@@ -586,8 +619,25 @@ struct TileCtx {
     bool aligned;
     const uint32_t *Qe, *Qc;
     const uint16_t *Sj;
+    const uint32_t *stash;  // first 32 bytes of every chunk (valid when aligned and >= 32 bytes)
+    const uint32_t *ext;    // eager-completion entries, kExt per chunk
     DevStats *stats;
 };
+
+// Look up an eager-completion entry of chunk c for state st: returns the slot (or -1) and delta.
+__device__ __forceinline__ int ext_lookup(const uint32_t *ext, uint32_t c, uint32_t st, int32_t &delta)
+{
+    const uint32_t *ex = ext + c * kExt;
+#pragma unroll
+    for (int q = 0; q < kExt; q++) {
+        const uint32_t v = ex[q];
+        if ((v & 0xFFFFu) == st) {
+            delta = (int32_t)v >> 20;
+            return (int)((v >> 16) & 0xFu);
+        }
+    }
+    return -1;
+}
 
 // a8: resolve a broken slot.  The run is in state `st` when entering chunk c of the tile, with
 // count n so far.  Re-execute chunk c from st in lockstep with the chunk's speculated chains
@@ -599,6 +649,22 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
                         uint32_t &out_n)
 {
     for (;;) {
+        {   // eager completion already ran this state into one of the chunk's chains
+            int32_t dl;
+            const int l = ext_lookup(t.ext, c, st, dl);
+            if (l >= 0) {
+                n += (uint32_t)dl + t.Qc[c * K + l];
+                const uint32_t x = t.Qe[c * K + l];
+                if ((x >> 16) == COMPLETE) {
+                    out_st = x & 0xFFFFu;
+                    out_n = n;
+                    return;
+                }
+                st = x & 0xFFFFu;
+                c = x >> 16;
+                continue;
+            }
+        }
         const uint64_t b = t.tile_base + (uint64_t)c * t.chunk;
         const uint64_t e = min(b + t.chunk, t.len);
         uint32_t y[K], cy[K];
@@ -625,6 +691,15 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
                     cyc = cy[l];
                 }
         };
+        if (t.aligned && e - b >= 32) {
+            // the chunk's first 32 bytes were stashed in smem by its owner during the local phase:
+            // the usual early exit never touches global memory
+#pragma unroll 1
+            for (int q = 0; q < 32 && conv < 0; q++) {
+                one((t.stash[c * 8 + (q >> 2)] >> (8 * (q & 3))) & 0xFFu);
+                pos++;
+            }
+        }
         if (t.aligned) {
             while (conv < 0 && pos + 16 <= e) {
                 const uint4 v = ldg128(t.in + pos);
@@ -696,6 +771,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
     uint32_t *wC = reinterpret_cast<uint32_t *>(smem + L.wc);
     uint32_t *wI = reinterpret_cast<uint32_t *>(smem + L.wi);
     uint32_t &s_tile = *reinterpret_cast<uint32_t *>(smem + L.misc);
+    uint32_t *Ext = reinterpret_cast<uint32_t *>(smem + L.ext);
 
     const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
     const unsigned long long start_count = p.start_dev ? p.start_dev->count : 0ull;
@@ -716,6 +792,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
 
         // ---- a3: speculated start set
         uint32_t S[K];
+        uint32_t cprev = 0, nimg_prev = 0;
         if (first_chunk && !p.keyed) {
 #pragma unroll
             for (int s = 0; s < K; s++) S[s] = s == 0 ? start_state : NOSTATE;
@@ -723,7 +800,9 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
             uint32_t c = 0;
             if (first_chunk) c = p.halo_byte;
             else if (!empty) c = __ldg(p.in + b - 1);
-            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
+            cprev = c;
+            nimg_prev = empty ? 0u : (uint32_t)__ldg(p.nimg + c);
+            const uint32_t ni = min(nimg_prev, ksel);
 #pragma unroll
             for (int s = 0; s < K; s++) S[s] = (!empty && (uint32_t)s < ni) ? (uint32_t)__ldg(p.lb + c * KMAX + s) : NOSTATE;
         }
@@ -739,12 +818,64 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
             acc[s] = 0;
             accf[s] = 0;
         }
-        if (!empty && e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf);
+        if (!empty && e > b)
+            local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf,
+                           reinterpret_cast<uint32_t *>(smem + L.stash) + j * 8);
         uint32_t eob[K], cnt[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
             eob[s] = S[s] == NOSTATE ? (ABSENT << 16) : (tb.state_of(cur[s]) | (COMPLETE << 16));
             cnt[s] = tb.count_of(acc[s], accf[s], cur[s], empty ? 0 : e - b);
+        }
+
+        // ---- NEXT-3 eager completion (bounded): the next image states of the look-back symbol
+        // beyond the k speculated ones run in lockstep with the k chains over the stashed first
+        // 32 bytes; a state that meets a chain is recorded as (state, slot, count delta).
+        {
+            uint32_t ent[kExt];
+#pragma unroll
+            for (int q = 0; q < kExt; q++) ent[q] = kExtNone;
+            const uint32_t first_ext = min(nimg_prev, ksel);
+            if (p.aligned && !empty && e - b >= 32 && nimg_prev > first_ext) {
+                const uint32_t *st32 = reinterpret_cast<const uint32_t *>(smem + L.stash) + j * 8;
+                uint32_t y[K], cy[K], u[kExt], cu[kExt];
+                bool live[kExt];
+#pragma unroll
+                for (int l = 0; l < K; l++) {
+                    y[l] = S[l] == NOSTATE ? 0u : S[l];
+                    cy[l] = 0;
+                }
+                int nlive = 0;
+#pragma unroll
+                for (int q = 0; q < kExt; q++) {
+                    live[q] = first_ext + q < nimg_prev;
+                    u[q] = live[q] ? (uint32_t)__ldg(p.lb + cprev * KMAX + first_ext + q) : 0u;
+                    cu[q] = 0;
+                    nlive += live[q];
+                }
+#pragma unroll 1
+                for (int pos = 0; pos < 32 && nlive > 0; pos++) {
+                    const uint32_t byte = (st32[pos >> 2] >> (8 * (pos & 3))) & 0xFFu;
+                    const typename TB::Row r = tb.row(byte);
+#pragma unroll
+                    for (int l = 0; l < K; l++) y[l] = tb.apply(r, y[l], cy[l]);
+#pragma unroll
+                    for (int q = 0; q < kExt; q++) {
+                        if (!live[q]) continue;
+                        u[q] = tb.apply(r, u[q], cu[q]);
+#pragma unroll
+                        for (int l = 0; l < K; l++)
+                            if (live[q] && S[l] != NOSTATE && y[l] == u[q]) {
+                                live[q] = false;
+                                nlive--;
+                                const uint32_t key = (uint32_t)__ldg(p.lb + cprev * KMAX + first_ext + q);
+                                ent[q] = key | ((uint32_t)l << 16) | (((cu[q] - cy[l]) & 0xFFFu) << 20);
+                            }
+                    }
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < kExt; q++) Ext[j * kExt + q] = ent[q];
         }
         bool ident = empty;
 
@@ -753,7 +884,8 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
         atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 40, (unsigned long long)(t_local1 - t_local0));
 #endif
         // ---- a5: warp stage (chunks warp*32 .. warp*32+31)
-        warp_suffix_scan<K>(S, eob, cnt, ident, (uint32_t)warp * 32, 1);
+        __syncwarp();  // the lanes' eager-completion entries are read by the scan
+        warp_suffix_scan<K>(S, eob, cnt, ident, (uint32_t)warp * 32, 1, Ext);
 
         // ---- a6: block stage
         if (lane == 0) {
@@ -781,7 +913,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
 #pragma unroll
                 for (int s = 0; s < K; s++) S2[s] = NOSTATE, e2[s] = ABSENT << 16, c2[s] = 0;
             }
-            warp_suffix_scan<K>(S2, e2, c2, id2, 0, 32);
+            warp_suffix_scan<K>(S2, e2, c2, id2, 0, 32, Ext);
             __syncwarp();
             if (lane < W) {
 #pragma unroll
@@ -800,7 +932,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
                 er[s] = wE[(warp + 1) * K + s];
                 cr[s] = wC[(warp + 1) * K + s];
             }
-            compose<K>(eob, cnt, Sr, er, cr, (uint32_t)(warp + 1) * 32);
+            compose<K>(eob, cnt, Sr, er, cr, (uint32_t)(warp + 1) * 32, Ext);
         }
 #pragma unroll
         for (int s = 0; s < K; s++) {
@@ -831,6 +963,8 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
         t.Qe = Qe;
         t.Qc = Qc;
         t.Sj = Sj;
+        t.stash = reinterpret_cast<const uint32_t *>(smem + L.stash);
+        t.ext = Ext;
         t.stats = p.stats;
 
         // a8 (tile candidates): resolve the broken slots of the tile aggregate Q_0 so that the

@@ -34,14 +34,16 @@ METRIC = "input GB/s (final state+accept count bit-exact)"
 
 # ----------------------------------------------------------------------------- workloads
 def make_workload(args):
-    """Returns dict(dfa, k, name, total_bytes, fill(dev_ptr, lo, n), host(lo, n) -> np.ndarray)."""
+    """Returns dict(dfa, k, name, total, bits, and either data (host array, generated once) or
+    fill(dev_ptr, lo, n, stream) + host(lo, n) for the counter-based C5 stream)."""
     from fsmgen import dfas, streams
 
     seed = streams.MASTER_SEED
     cfg = args.config
+    gib = args.size_gib
     if cfg == "c5":
         d = dfas.random_dfa(args.n_states, args.m, seed=seed + 5)
-        total = int(args.size_gib * GiB)
+        total = int((gib or 64.0) * GiB)
         sseed = seed + 5
 
         def fill(ptr, lo, n, stream=0):
@@ -60,13 +62,37 @@ def make_workload(args):
             return out[:n]
 
         name = (f"C5 random DFA N={args.n_states} m={args.m} (|image(c)|=m), spec-{args.k}, "
-                f"{args.size_gib:g} GiB i.i.d. bytes")
+                f"{total / GiB:g} GiB i.i.d. bytes")
         return dict(dfa=d, k=args.k, name=name, total=total, fill=fill, host=host, bits=False)
     if cfg == "c1":
         d = dfas.c_comment(True)
-        total = 1 << 20
+        total = int((gib or 1.0 / 1024) * GiB)
         data = streams.c_source(total, seed=seed + 1)
-        return dict(dfa=d, k=1, name="C1 C-comment FSM (Fig. 1, 4 states x 3 classes) 1 MiB synthetic C, spec-1",
+        k = args.k_override or 1
+        return dict(dfa=d, k=k, name=f"C1 C-comment FSM (Fig. 1, 4 states x 3 classes) on {total} B synthetic C, spec-{k}",
+                    total=total, data=data, bits=False)
+    if cfg == "c2":
+        w = dfas.zipf_weights(256, seed=seed + 2)
+        d, codes = dfas.huffman(w.tolist())
+        nbytes = int((gib or 1.0) * GiB)
+        data, _ = streams.huffman_stream(codes, w, nbytes * 8, seed + 2)
+        k = args.k_override or 4
+        return dict(dfa=d, k=k, name=f"C2 Huffman decoder (Zipf-1, 256 symbols, {d.n_states} states, bit alphabet) "
+                    f"on {nbytes / GiB:g} GiB encoded bitstream, spec-{k}", total=nbytes, data=data, bits=True)
+    if cfg == "c3":
+        pats = dfas.snort_patterns(args.ac_states, seed=seed + 3)
+        d = dfas.aho_corasick(pats)
+        total = int((gib or 4.0) * GiB)
+        data = streams.ac_payload(total, seed + 3, pats)
+        k = args.k_override or 1
+        return dict(dfa=d, k=k, name=f"C3 Snort-style Aho-Corasick DFA ({d.n_states} states, 256 symbols) on "
+                    f"{total / GiB:g} GiB synthetic packet payloads, spec-{k}", total=total, data=data, bits=False)
+    if cfg == "c4":
+        d = dfas.html_tokenizer()
+        total = int((gib or 8.0) * GiB)
+        data = streams.html_bytes(total, seed + 4)
+        k = args.k_override or 1
+        return dict(dfa=d, k=k, name=f"C4 HTML tokenizer (38 states) on {total / GiB:g} GiB synthetic HTML, spec-{k}",
                     total=total, data=data, bits=False)
     raise SystemExit(f"unknown config {cfg}")
 
@@ -174,11 +200,13 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="c5", choices=["c5", "c1"])
+    ap.add_argument("--config", default="c5", choices=["c1", "c2", "c3", "c4", "c5"])
+    ap.add_argument("--k-override", type=int, default=0, help="k for c1-c4 (c5 uses --k)")
+    ap.add_argument("--ac-states", type=int, default=1024, help="c3: minimum Aho-Corasick states (1024 / 4096)")
     ap.add_argument("--n-states", type=int, default=8)
     ap.add_argument("--m", type=int, default=2)
     ap.add_argument("--k", type=int, default=2)
-    ap.add_argument("--size-gib", type=float, default=64.0)
+    ap.add_argument("--size-gib", type=float, default=0.0, help="input size (default: the config's)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--variant", type=int, default=-1)
@@ -210,6 +238,7 @@ def main():
     lo = total * rank // world // 32 * 32
     hi = total if rank == world - 1 else total * (rank + 1) // world // 32 * 32
     n = hi - lo
+    nsym = n * 8 if w["bits"] else n   # the library counts symbols: bits in bit mode
     buf = torch.empty(n + 64, dtype=torch.uint8, device=dev)
     halo = torch.zeros(32, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
@@ -233,9 +262,9 @@ def main():
 
     def step():
         if world == 1:
-            f.run_spec_k_async(buf.data_ptr(), n, k, res.data_ptr())
+            f.run_spec_k_async(buf.data_ptr(), nsym, k, res.data_ptr())
             return None
-        return run_sharded(f, buf.data_ptr(), n, halo.data_ptr() if rank else None, k, d.start, device=dev)
+        return run_sharded(f, buf.data_ptr(), nsym, halo.data_ptr() if rank else None, k, d.start, device=dev)
 
     # parity gate on the bench's own launch configuration: the prefix sample the oracle also times
     for _ in range(args.warmup):
@@ -264,7 +293,7 @@ def main():
     step_s = float(t.item())
     st = f.stats() if world == 1 else {}
     if world == 1:
-        f.run_spec_k(buf.data_ptr(), n, k)
+        f.run_spec_k(buf.data_ptr(), nsym, k)
         st = f.stats()
     r = res.cpu().numpy().view(np.uint32)
     final = (int(r[0]), int(r[2]) | (int(r[3]) << 32)) if world == 1 else out
@@ -289,7 +318,7 @@ def main():
                 for i in range(max(1, min(args.steps, 3)) + 1):
                     torch.cuda.synchronize()
                     t0 = time.perf_counter()
-                    got = f.run_spec_k_host(hbuf.data_ptr(), n, k)
+                    got = f.run_spec_k_host(hbuf.data_ptr(), nsym, k)
                     dt = time.perf_counter() - t0
                     if i:
                         et.append(dt)
@@ -332,11 +361,11 @@ def main():
     if not args.no_ablation and world == 1:
         # internal ablation: the paper's sequential merge (Fig. 4a) on the same input and chains
         f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_SEQUENTIAL)
-        f.run_spec_k_async(buf.data_ptr(), n, k, res.data_ptr())
+        f.run_spec_k_async(buf.data_ptr(), nsym, k, res.data_ptr())
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        f.run_spec_k_async(buf.data_ptr(), n, k, res.data_ptr())
+        f.run_spec_k_async(buf.data_ptr(), nsym, k, res.data_ptr())
         e1.record(stream)
         torch.cuda.synchronize()
         ts = e0.elapsed_time(e1) / 1e3
@@ -353,7 +382,7 @@ def main():
             pass
         cb = cpu_oracle_rate(w, budget_s=12.0)
         # parity on the sampled prefix: the GPU runs the same prefix in the bench's configuration
-        gp = f.run_spec_k(buf.data_ptr(), cb["bytes"], k)
+        gp = f.run_spec_k(buf.data_ptr(), cb["bytes"] * (8 if w["bits"] else 1), k)
         line["cpu_baseline"] = {"value": round(cb["gbs"], 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
                                 "sample": f"first {cb['bytes']} bytes of the workload ({cb['seconds']:.1f} s)"}
         line["parity_sample"] = {"bytes": cb["bytes"], "ok": gp == cb["result"]}

@@ -48,6 +48,14 @@ def host_lib() -> ctypes.CDLL:
         lib.fsmgen_word.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
         lib.fsmgen_fill.restype = None
         lib.fsmgen_fill.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64]
+        lib.fsmgen_html_block.restype = None
+        lib.fsmgen_html_block.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64]
+        lib.fsmgen_ac_block.restype = None
+        lib.fsmgen_ac_block.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64,
+                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32]
+        lib.fsmgen_huffman.restype = ctypes.c_uint64
+        lib.fsmgen_huffman.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p,
+                                       ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p]
         _host = lib
     return _host
 

@@ -203,3 +203,78 @@ def random_dfa(n_states: int, m: int, seed: int, alphabet: int = 256) -> DFA:
         t[:, c] = col
     acc = np.array([streams.word(seed, s) % 4 == 0 for s in range(n_states)], dtype=np.uint8)
     return DFA(t, 0, acc, False, f"random_{n_states}_{m}")
+
+
+# ---------------------------------------------------------------------------------------------
+# W5: HTML tokenizer with exactly 38 states (PAPER.md:269 gives only "38 states, 128 inputs"; the
+# FSM itself is our construction, reading A17).  Simplified WHATWG tokenizer; bytes >= 0x80 behave
+# as letters.  Accepting states are the token-complete "emit" states, so the accept count is the
+# number of tokens: tags, comments, declarations, character references and text runs (a text run
+# is counted by the '<' that ends it).
+HTML_STATES = [
+    "Data", "Text", "TextEmit", "TagOpen", "EndTagOpen", "TagName", "EndTagName", "BeforeAttrName",
+    "AttrName", "AfterAttrName", "BeforeAttrValue", "AttrValueDQ", "AttrValueSQ", "AttrValueUnq",
+    "AfterAttrValueQuoted", "SelfClosingStart", "TagEmit", "MarkupDeclOpen", "CommentStartDash",
+    "CommentStart", "Comment", "CommentEndDash", "CommentEnd", "CommentEmit", "DocD", "DocO", "DocC",
+    "DocT", "DocY", "DocP", "DocE", "DoctypeBody", "DoctypeEmit", "CharRef", "CharRefNamed",
+    "CharRefNumeric", "CharRefHex", "CharRefEmit"]
+HTML_ACCEPT = ("TextEmit", "TagEmit", "CommentEmit", "DoctypeEmit", "CharRefEmit")
+
+
+def html_tokenizer() -> DFA:
+    S = {n: i for i, n in enumerate(HTML_STATES)}
+    assert len(S) == 38
+    ws = set(b" \t\n\r\f")
+    letters = set(range(ord("a"), ord("z") + 1)) | set(range(ord("A"), ord("Z") + 1)) | set(range(0x80, 0x100))
+    digits = set(range(ord("0"), ord("9") + 1))
+    hexd = digits | set(b"abcdefABCDEF")
+    t = np.zeros((38, 256), dtype=np.uint32)
+
+    def setrow(state, default, rules):
+        r = t[S[state]]
+        r[:] = S[default]
+        for chars, dst in rules:
+            for c in chars:
+                r[c] = S[dst]
+
+    lt, gt, sl, ex, da, eq = ord("<"), ord(">"), ord("/"), ord("!"), ord("-"), ord("=")
+    dq, sq, am, hs, sc = ord('"'), ord("'"), ord("&"), ord("#"), ord(";")
+    data_rules = [([lt], "TagOpen"), ([am], "CharRef")]
+    for st in ("Data", "TagEmit", "CommentEmit", "DoctypeEmit", "CharRefEmit"):
+        setrow(st, "Text", data_rules)
+    setrow("Text", "Text", [([lt], "TextEmit"), ([am], "CharRef")])
+    for st in ("TagOpen", "TextEmit"):
+        setrow(st, "Text", [(letters, "TagName"), ([sl], "EndTagOpen"), ([ex], "MarkupDeclOpen"), ([lt], "TagOpen")])
+    setrow("EndTagOpen", "Text", [(letters, "EndTagName"), ([gt], "Data")])
+    setrow("TagName", "TagName", [(ws, "BeforeAttrName"), ([sl], "SelfClosingStart"), ([gt], "TagEmit")])
+    setrow("EndTagName", "EndTagName", [([gt], "TagEmit")])
+    setrow("BeforeAttrName", "AttrName", [(ws, "BeforeAttrName"), ([sl], "SelfClosingStart"), ([gt], "TagEmit")])
+    setrow("AttrName", "AttrName", [(ws, "AfterAttrName"), ([sl], "SelfClosingStart"), ([eq], "BeforeAttrValue"),
+                                    ([gt], "TagEmit")])
+    setrow("AfterAttrName", "AttrName", [(ws, "AfterAttrName"), ([sl], "SelfClosingStart"),
+                                         ([eq], "BeforeAttrValue"), ([gt], "TagEmit")])
+    setrow("BeforeAttrValue", "AttrValueUnq", [(ws, "BeforeAttrValue"), ([dq], "AttrValueDQ"),
+                                               ([sq], "AttrValueSQ"), ([gt], "TagEmit")])
+    setrow("AttrValueDQ", "AttrValueDQ", [([dq], "AfterAttrValueQuoted")])
+    setrow("AttrValueSQ", "AttrValueSQ", [([sq], "AfterAttrValueQuoted")])
+    setrow("AttrValueUnq", "AttrValueUnq", [(ws, "BeforeAttrName"), ([gt], "TagEmit")])
+    setrow("AfterAttrValueQuoted", "AttrName", [(ws, "BeforeAttrName"), ([sl], "SelfClosingStart"), ([gt], "TagEmit")])
+    setrow("SelfClosingStart", "AttrName", [([gt], "TagEmit"), (ws, "BeforeAttrName")])
+    setrow("MarkupDeclOpen", "DoctypeBody", [([da], "CommentStartDash"), (b"Dd", "DocD"), ([gt], "DoctypeEmit")])
+    setrow("CommentStartDash", "DoctypeBody", [([da], "CommentStart"), ([gt], "DoctypeEmit")])
+    setrow("CommentStart", "Comment", [([da], "CommentEndDash"), ([gt], "CommentEmit")])
+    setrow("Comment", "Comment", [([da], "CommentEndDash")])
+    setrow("CommentEndDash", "Comment", [([da], "CommentEnd")])
+    setrow("CommentEnd", "Comment", [([gt], "CommentEmit"), ([da], "CommentEnd")])
+    for a, b, nxt in (("DocD", "Oo", "DocO"), ("DocO", "Cc", "DocC"), ("DocC", "Tt", "DocT"),
+                      ("DocT", "Yy", "DocY"), ("DocY", "Pp", "DocP"), ("DocP", "Ee", "DocE")):
+        setrow(a, "DoctypeBody", [(b.encode(), nxt), ([gt], "DoctypeEmit")])
+    setrow("DocE", "DoctypeBody", [([gt], "DoctypeEmit")])
+    setrow("DoctypeBody", "DoctypeBody", [([gt], "DoctypeEmit")])
+    setrow("CharRef", "Text", [([hs], "CharRefNumeric"), (letters, "CharRefNamed"), ([lt], "TagOpen")])
+    setrow("CharRefNamed", "Text", [(letters | digits, "CharRefNamed"), ([sc], "CharRefEmit"), ([lt], "TagOpen")])
+    setrow("CharRefNumeric", "Text", [(b"xX", "CharRefHex"), (digits, "CharRefNumeric"), ([sc], "CharRefEmit"),
+                                      ([lt], "TagOpen")])
+    setrow("CharRefHex", "Text", [(hexd, "CharRefHex"), ([sc], "CharRefEmit"), ([lt], "TagOpen")])
+    acc = np.array([1 if n in HTML_ACCEPT else 0 for n in HTML_STATES], dtype=np.uint8)
+    return DFA(t, S["Data"], acc, False, "html38")

@@ -162,3 +162,68 @@ def huffman_bits(codes: list[str], probs: np.ndarray, n_bits: int, seed: int) ->
         b += 1
     allbits = np.concatenate(out_bits) if out_bits else np.zeros(0, np.uint8)
     return np.packbits(allbits), complete
+
+
+# ----------------------------------------------------------------------------------------------
+# Large structured inputs through the C generators (block-seeded, generated on all host cores)
+def _blocks_parallel(fn, n: int, out: np.ndarray | None = None) -> np.ndarray:
+    import concurrent.futures as cf
+    import os
+
+    if out is None:
+        out = np.empty(n, dtype=np.uint8)
+    nb = (n + BLOCK - 1) // BLOCK
+    with cf.ThreadPoolExecutor(os.cpu_count()) as ex:
+        list(ex.map(lambda b: fn(out[b * BLOCK:], min(BLOCK, n - b * BLOCK), b), range(nb)))
+    return out[:n]
+
+
+def html_bytes(n: int, seed: int, out: np.ndarray | None = None) -> np.ndarray:
+    """C4 input: synthetic HTML documents (nested tags from a 40-tag vocabulary, depth <= 8, 0-4
+    attributes with double/single/unquoted values, word text runs, ~3 % comments, ~1 % entities,
+    one DOCTYPE per document), 1 MiB blocks."""
+    lib = _native.host_lib()
+    return _blocks_parallel(lambda o, m, b: lib.fsmgen_html_block(o.ctypes.data, m, seed, b), n, out)
+
+
+def ac_payload(n: int, seed: int, patterns: list[bytes], out: np.ndarray | None = None) -> np.ndarray:
+    """C3 input: packet payloads of U[64,1500] bytes, 75 % content-set bytes, 25 % uniform, a
+    random pattern planted with probability 1e-3 per position, 1 MiB blocks."""
+    lib = _native.host_lib()
+    pats = np.frombuffer(b"".join(patterns), dtype=np.uint8).copy()
+    offs = np.zeros(len(patterns) + 1, dtype=np.uint32)
+    offs[1:] = np.cumsum([len(p) for p in patterns])
+    return _blocks_parallel(lambda o, m, b: lib.fsmgen_ac_block(o.ctypes.data, m, seed, b, pats.ctypes.data,
+                                                                offs.ctypes.data, len(patterns)), n, out)
+
+
+def _alias(probs: np.ndarray):
+    n = probs.size
+    p = probs * n / probs.sum()
+    prob = np.zeros(n, np.float64)
+    alias = np.zeros(n, np.uint32)
+    small = [i for i in range(n) if p[i] < 1.0]
+    large = [i for i in range(n) if p[i] >= 1.0]
+    while small and large:
+        s, l = small.pop(), large.pop()
+        prob[s] = p[s]
+        alias[s] = l
+        p[l] = p[l] + p[s] - 1.0
+        (small if p[l] < 1.0 else large).append(l)
+    for i in large + small:
+        prob[i] = 1.0
+        alias[i] = i
+    return np.minimum(np.floor(prob * 2.0 ** 32), 2.0 ** 32 - 1).astype(np.uint32), alias
+
+
+def huffman_stream(codes: list[str], weights: np.ndarray, n_bits: int, seed: int) -> tuple[np.ndarray, int]:
+    """C2 input: i.i.d. symbols (alias method over ``weights``) Huffman-encoded MSB-first, cut at
+    exactly n_bits bits.  Returns (packed bytes, number of complete codewords)."""
+    lib = _native.host_lib()
+    prob, alias = _alias(np.asarray(weights, dtype=np.float64))
+    code = np.array([int(c, 2) for c in codes], dtype=np.uint32)
+    clen = np.array([len(c) for c in codes], dtype=np.uint8)
+    out = np.zeros((n_bits + 7) // 8 + 8, dtype=np.uint8)
+    nsym = lib.fsmgen_huffman(out.ctypes.data, n_bits, seed, prob.ctypes.data, alias.ctypes.data, len(codes),
+                              code.ctypes.data, clen.ctypes.data)
+    return out[:(n_bits + 7) // 8], int(nsym)

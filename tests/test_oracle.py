@@ -351,3 +351,38 @@ def test_div7_hit_rate_linear_in_k():
     for k, rate in zip((1, 2, 4, 7), rates):
         assert abs(rate - k / 7) < 0.06, (k, rate)
     assert rates[-1] == 1.0
+
+
+def test_html_tokenizer_structure_and_snippets(golden):
+    d = dfas.html_tokenizer()
+    assert d.n_states == 38 and d.alphabet == 256          # PAPER.md:269 (38 states)
+    assert (d.table[:, 0x80:] == d.table[:, [ord("g")]]).all()   # bytes >= 0x80 act as letters (A17)
+    for case in golden["html_snippets"]["cases"]:
+        q, n = seq.run(d, np.frombuffer(case["html"].encode(), np.uint8))
+        assert (dfas.HTML_STATES[q], n) == (case["final"], case["count"]), case
+
+
+def test_c_generators_round_trip():
+    """Generator pins: the C Huffman encoder's complete-codeword count equals the decoder DFA's
+    accept count (root visits); AC payload accept count equals naive multi-pattern search; HTML
+    blocks are deterministic per (seed, block)."""
+    w = dfas.zipf_weights(256, seed=3)
+    d, codes = dfas.huffman(w.tolist())
+    n_bits = 8 * 100_000 + 3
+    data, nsym = streams.huffman_stream(codes, w, n_bits, seed=9)
+    assert seq.run(d, data, n_bits)[1] == nsym
+    pats = dfas.snort_patterns(200, seed=4)
+    ad = dfas.aho_corasick(pats)
+    pay = streams.ac_payload(1 << 18, 5, pats)
+    text = pay.tobytes()
+    ends = set()
+    for p in pats:
+        i = text.find(p)
+        while i >= 0:
+            ends.add(i + len(p))
+            i = text.find(p, i + 1)
+    assert seq.run(ad, pay)[1] == len(ends) > 0
+    h1 = streams.html_bytes(3 << 20, 11)
+    h2 = streams.html_bytes(3 << 20, 11)
+    assert (h1 == h2).all() and h1[:15].tobytes() == b"<!DOCTYPE html>"
+    assert seq.run(dfas.html_tokenizer(), h1)[1] > 10000

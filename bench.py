@@ -188,7 +188,7 @@ def run_reference(args, w):
 
 
 def config_json(args, w):
-    return {"workload": w["name"], "input_bytes": w["total"], "k": w["k"],
+    return {"workload": w["name"], "input_bytes": w["total"], "k": w["k"], "lookback_len": w.get("lookback"),
             "n_states": int(w["dfa"].n_states), "parallelism": f"shard{args.gpus}",
             "l2": "input >> L2 (126 MB), no flush needed" if w["total"] > 4 * 126e6 else "L2 flushed between steps"}
 
@@ -210,6 +210,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--variant", type=int, default=-1)
+    ap.add_argument("--lookback", type=int, default=-1,
+                    help="look-back window bytes (R7; -1 = the config's default: c5 0, c1/c4 64, c2/c3 32)")
     ap.add_argument("--chunk", type=int, default=0)
     ap.add_argument("--no-ablation", action="store_true",
                     help="skip the sequential-merge ablation run (Fig. 4a, SURVEY 8.a11)")
@@ -254,8 +256,9 @@ def main():
 
     f = FSM.from_dfa(d)
     f.set_stream(stream.cuda_stream)
-    if args.variant >= 0 or args.chunk:
-        f.set_options(variant=args.variant, chunk_bytes=args.chunk)
+    lookback = args.lookback if args.lookback >= 0 else {"c5": 0, "c1": 64, "c4": 64, "c2": 32, "c3": 32}[args.config]
+    w["lookback"] = lookback
+    f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback)
     res = torch.zeros(4, dtype=torch.int32, device=dev)
     small = total < 4 * 126_000_000
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if small else None
@@ -360,7 +363,8 @@ def main():
     }
     if not args.no_ablation and world == 1:
         # internal ablation: the paper's sequential merge (Fig. 4a) on the same input and chains
-        f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_SEQUENTIAL)
+        f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_SEQUENTIAL,
+                      lookback_len=lookback)
         f.run_spec_k_async(buf.data_ptr(), nsym, k, res.data_ptr())
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -371,7 +375,8 @@ def main():
         ts = e0.elapsed_time(e1) / 1e3
         r2 = res.cpu().numpy().view(np.uint32)
         same = (int(r2[0]), int(r2[2]) | (int(r2[3]) << 32)) == final
-        f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_PARALLEL)
+        f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_PARALLEL,
+                      lookback_len=lookback)
         line["ablation"] = {"sequential_merge_gbs": round(n / ts / 1e9, 3),
                             "parallel_over_sequential": round(ts / step_s, 2), "same_result": same,
                             "paper_v100_context": "2.02-6.74x (P:11, P:53)"}

@@ -126,6 +126,9 @@ typedef struct {
     int32_t variant;            /* FSM_VARIANT_*; FSM_VARIANT_AUTO = by state count */
     uint32_t merge;             /* FSM_MERGE_* */
     uint32_t ctas_per_sm;       /* cap on resident CTAs per SM for the persistent grid; 0 = max */
+    uint32_t lookback_len;      /* look-back: 0 or 1 = the byte before the chunk; 32..1024 (multiple
+                                   of 32) = run the image of the byte before a window of that many bytes
+                                   through the window and rank the reached states by multiplicity */
 } fsm_options;
 
 int fsm_set_options(fsm_t *f, const fsm_options *opt);
@@ -139,7 +142,7 @@ typedef struct {
     uint64_t reexec_chunks;     /* chunk re-executions (true-path and tile-candidate paths) */
     uint64_t reexec_symbols;    /* bytes consumed by re-executions (early exit on convergence) */
     uint64_t boundary_misses;   /* tile-boundary misses resolved after the look-back */
-    uint32_t chunk_bytes, threads_per_tile, variant, k_slots;
+    uint32_t chunk_bytes, threads_per_tile, variant, k_slots, lookback_len;
 } fsm_stats;
 
 int fsm_get_stats(const fsm_t *f, fsm_stats *s);

@@ -328,11 +328,13 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_H8) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
+    if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
     f->opt.chunk_bytes = o->chunk_bytes;            // 0 = adaptive
     f->opt.threads_per_tile = o->threads_per_tile;  // 0 = auto
     f->opt.variant = o->variant;
     f->opt.merge = o->merge;
     f->opt.ctas_per_sm = o->ctas_per_sm;
+    f->opt.lookback_len = o->lookback_len;
     return FSM_OK;
 }
 
@@ -432,6 +434,7 @@ static int launch_run(fsm *f, const RunSpec &r)
     p.chunk = chunk;
     p.ntiles = ntiles;
     p.k = r.k;
+    p.lookback = f->opt.lookback_len > 1 ? f->opt.lookback_len : 0;
     p.aligned = ((uintptr_t)r.in & 31) == 0;
     p.table = f->d_img[var];
     p.n_states = f->dfa.n;
@@ -482,6 +485,7 @@ static int launch_run(fsm *f, const RunSpec &r)
     f->last.threads_per_tile = T;
     f->last.variant = var;
     f->last.k_slots = K;
+    f->last.lookback_len = p.lookback;
     return FSM_OK;
 }
 
@@ -521,6 +525,7 @@ static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T)
     f->last.threads_per_tile = T;
     f->last.variant = var;
     f->last.k_slots = K;
+    f->last.lookback_len = p.lookback;
     return FSM_OK;
 }
 

@@ -31,16 +31,8 @@ __global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb
     const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
     for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nch; g += (uint64_t)gridDim.x * blockDim.x) {
         const uint64_t b = g * p.chunk, e = min(b + p.chunk, p.len);
-        uint32_t S[K];
-        if (g == 0) {
-#pragma unroll
-            for (int s = 0; s < K; s++) S[s] = s == 0 ? start_state : NOSTATE;
-        } else {
-            const uint32_t c = __ldg(p.in + b - 1);
-            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), p.k);
-#pragma unroll
-            for (int s = 0; s < K; s++) S[s] = (uint32_t)s < ni ? (uint32_t)__ldg(p.lb + c * KMAX + s) : NOSTATE;
-        }
+        uint32_t S[K], Xc[kExt];
+        speculate<K>(tb, p, b, g == 0, false, start_state, S, Xc);
         uint32_t cur[K], acc[K], accf[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {

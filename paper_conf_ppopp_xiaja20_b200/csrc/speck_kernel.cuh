@@ -516,6 +516,99 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
     }
 }
 
+
+// ----------------------------------------------------------------- a3: look-back speculation --
+// Candidate start states of the chunk starting at byte b, ranked.  Depth 1 (lookback < 32): the
+// image of the preceding byte ranked by preimage count (A5; host table LB).  Window
+// (lookback = Lw >= 32, multiple of 32): the image of x[b-Lw-1] is run through the Lw bytes
+// before the chunk and the reached states are ranked by multiplicity (how many image states
+// reach each), ties to the smaller id -- the same rule one level deeper (reading R7).  If the
+// window would reach before the start of a known-start run, the single exact state is used.
+// Returns S (top k, NOSTATE-padded), X (the next kExt candidates, for eager completion).
+template <int K, class TB>
+__device__ __forceinline__ void speculate(const TB &tb, const Params &p, uint64_t b, bool first_chunk, bool empty,
+                                          uint32_t start_state, uint32_t (&S)[K], uint32_t (&X)[kExt])
+{
+#pragma unroll
+    for (int s = 0; s < K; s++) S[s] = NOSTATE;
+#pragma unroll
+    for (int q = 0; q < kExt; q++) X[q] = NOSTATE;
+    if (empty) return;
+    if (first_chunk && !p.keyed) {
+        S[0] = start_state;
+        return;
+    }
+    const uint32_t ksel = p.k;
+    const uint32_t Lw = p.lookback;
+    if (!first_chunk && Lw >= 32 && p.aligned && b >= Lw + 1) {
+        const uint32_t c0 = __ldg(p.in + b - Lw - 1);
+        const uint32_t ni = __ldg(p.nimg + c0);
+        uint32_t y[KMAX];
+#pragma unroll
+        for (int i = 0; i < KMAX; i++) y[i] = (uint32_t)__ldg(p.lb + c0 * KMAX + ((uint32_t)i < ni ? i : 0));
+        for (uint32_t o = 0; o < Lw; o += 32) {
+            const Bytes32 x = ldg256(p.in + b - Lw + o);
+#pragma unroll 1
+            for (int t = 0; t < 32; t++) {
+                const uint32_t byte = (x.w[t >> 2] >> (8 * (t & 3))) & 0xFFu;
+                const typename TB::Row r = tb.row(byte);
+                uint32_t dummy = 0;
+#pragma unroll
+                for (int i = 0; i < KMAX; i++) y[i] = tb.apply(r, y[i], dummy);
+            }
+        }
+        // rank the distinct reached states by multiplicity (over the ni real candidates)
+        uint32_t mult[KMAX];
+#pragma unroll
+        for (int i = 0; i < KMAX; i++) {
+            uint32_t m = 0;
+#pragma unroll
+            for (int j2 = 0; j2 < KMAX; j2++) m += ((uint32_t)j2 < ni && y[j2] == y[i]) ? 1u : 0u;
+            mult[i] = (uint32_t)i < ni ? m : 0u;
+        }
+        // selection: repeatedly take the best remaining (mult desc, id asc), then retire it
+#pragma unroll 1
+        for (uint32_t r = 0; r < (uint32_t)(K + kExt); r++) {
+            uint32_t bm = 0, bs = NOSTATE;
+#pragma unroll
+            for (int i = 0; i < KMAX; i++)
+                if (mult[i] > bm || (mult[i] == bm && mult[i] && y[i] < bs)) {
+                    bm = mult[i];
+                    bs = y[i];
+                }
+            if (!bm) break;
+#pragma unroll
+            for (int i = 0; i < KMAX; i++)
+                if (y[i] == bs) mult[i] = 0;
+            if (r < ksel) {
+#pragma unroll
+                for (int s = 0; s < K; s++)
+                    if ((uint32_t)s == r) S[s] = bs;
+            } else {
+#pragma unroll
+                for (int q = 0; q < kExt; q++)
+                    if ((uint32_t)q + ksel == r) X[q] = bs;
+            }
+        }
+        return;
+    }
+    if (!first_chunk && !p.keyed && Lw >= 32 && b < Lw + 1 && b > 0) {
+        // the window reaches the start of the run: run it exactly from the known start
+        uint32_t st = start_state, dummy = 0;
+        for (uint64_t t = 0; t < b; t++) st = tb.apply(tb.row(__ldg(p.in + t)), st, dummy);
+        S[0] = st;
+        return;
+    }
+    const uint32_t c = first_chunk ? p.halo_byte : (uint32_t)__ldg(p.in + b - 1);
+    const uint32_t ni = __ldg(p.nimg + c);
+#pragma unroll
+    for (int s = 0; s < K; s++)
+        if ((uint32_t)s < min(ni, ksel)) S[s] = (uint32_t)__ldg(p.lb + c * KMAX + s);
+#pragma unroll
+    for (int q = 0; q < kExt; q++)
+        if (ksel + q < ni) X[q] = (uint32_t)__ldg(p.lb + c * KMAX + ksel + q);
+}
+
 // --------------------------------------------------------- a5/a6: composition of mappings --
 // (L x R)[s]: a complete slot of L whose end state is a speculated start of R continues with R's
 // slot (which may itself be broken further on) and adds counts -- the membership check of
@@ -790,22 +883,9 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
         const bool empty = b >= p.len && !first_chunk;
         const uint64_t e = b >= p.len ? b : min(b + p.chunk, p.len);
 
-        // ---- a3: speculated start set
-        uint32_t S[K];
-        uint32_t cprev = 0, nimg_prev = 0;
-        if (first_chunk && !p.keyed) {
-#pragma unroll
-            for (int s = 0; s < K; s++) S[s] = s == 0 ? start_state : NOSTATE;
-        } else {
-            uint32_t c = 0;
-            if (first_chunk) c = p.halo_byte;
-            else if (!empty) c = __ldg(p.in + b - 1);
-            cprev = c;
-            nimg_prev = empty ? 0u : (uint32_t)__ldg(p.nimg + c);
-            const uint32_t ni = min(nimg_prev, ksel);
-#pragma unroll
-            for (int s = 0; s < K; s++) S[s] = (!empty && (uint32_t)s < ni) ? (uint32_t)__ldg(p.lb + c * KMAX + s) : NOSTATE;
-        }
+        // ---- a3: speculated start set (+ eager-completion candidates)
+        uint32_t S[K], Xc[kExt];
+        speculate<K>(tb, p, b, first_chunk, empty, start_state, S, Xc);
 
         // ---- a4: local processing
 #ifdef FSM_PHASE_TIMING
@@ -835,8 +915,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
             uint32_t ent[kExt];
 #pragma unroll
             for (int q = 0; q < kExt; q++) ent[q] = kExtNone;
-            const uint32_t first_ext = min(nimg_prev, ksel);
-            if (p.aligned && !empty && e - b >= 32 && nimg_prev > first_ext) {
+            if (p.aligned && !empty && e - b >= 32 && Xc[0] != NOSTATE) {
                 const uint32_t *st32 = reinterpret_cast<const uint32_t *>(smem + L.stash) + j * 8;
                 uint32_t y[K], cy[K], u[kExt], cu[kExt];
                 bool live[kExt];
@@ -848,8 +927,8 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
                 int nlive = 0;
 #pragma unroll
                 for (int q = 0; q < kExt; q++) {
-                    live[q] = first_ext + q < nimg_prev;
-                    u[q] = live[q] ? (uint32_t)__ldg(p.lb + cprev * KMAX + first_ext + q) : 0u;
+                    live[q] = Xc[q] != NOSTATE;
+                    u[q] = live[q] ? Xc[q] : 0u;
                     cu[q] = 0;
                     nlive += live[q];
                 }
@@ -868,8 +947,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
                             if (live[q] && S[l] != NOSTATE && y[l] == u[q]) {
                                 live[q] = false;
                                 nlive--;
-                                const uint32_t key = (uint32_t)__ldg(p.lb + cprev * KMAX + first_ext + q);
-                                ent[q] = key | ((uint32_t)l << 16) | (((cu[q] - cy[l]) & 0xFFFu) << 20);
+                                ent[q] = Xc[q] | ((uint32_t)l << 16) | (((cu[q] - cy[l]) & 0xFFFu) << 20);
                             }
                     }
                 }

@@ -57,6 +57,7 @@ struct Params {
     uint32_t chunk;                // bytes per chunk (multiple of 32)
     uint32_t ntiles;
     uint32_t k;                    // speculated states in use (<= template K)
+    uint32_t lookback;             // look-back window in bytes (0/1: the preceding byte only)
     uint32_t aligned;              // `in` is 32-byte aligned
     const void *table;             // variant image in global memory
     uint32_t n_states;             // internal states (incl. sink)

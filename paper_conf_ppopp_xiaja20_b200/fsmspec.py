@@ -30,14 +30,15 @@ EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_se
 
 class fsm_options(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
-                ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32)]
+                ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32),
+                ("lookback_len", ctypes.c_uint32)]
 
 
 class fsm_stats(ctypes.Structure):
     _fields_ = [("chunks", ctypes.c_uint64), ("tiles", ctypes.c_uint64), ("reexec_chunks", ctypes.c_uint64),
                 ("reexec_symbols", ctypes.c_uint64), ("boundary_misses", ctypes.c_uint64),
                 ("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
-                ("variant", ctypes.c_uint32), ("k_slots", ctypes.c_uint32)]
+                ("variant", ctypes.c_uint32), ("k_slots", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32)]
 
 
 class fsm_shard_map(ctypes.Structure):
@@ -174,8 +175,8 @@ class FSM:
         _check(lib().fsm_set_stream(self._h, s), "fsm_set_stream")
 
     def set_options(self, chunk_bytes: int = 0, threads_per_tile: int = 0, variant: int = FSM_VARIANT_AUTO,
-                    merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0) -> None:
-        o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm)
+                    merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0, lookback_len: int = 0) -> None:
+        o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm, lookback_len)
         _check(lib().fsm_set_options(self._h, ctypes.byref(o)), "fsm_set_options")
 
     def options(self) -> dict:

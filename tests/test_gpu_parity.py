@@ -234,3 +234,63 @@ def test_shard_maps_compose_and_fixup(G, k):
                 e, c = f.shard_fixup(shards[g], x)
             x, total = e, total + c
         assert (x, total) == exp
+
+
+# --------------------------------------------------------------------- look-back windows (R7)
+def _wl_cases():
+    pats = dfas.snort_patterns(300, seed=8)
+    w = dfas.zipf_weights(256, seed=4)
+    hd, codes = dfas.huffman(w.tolist())
+    hb, _ = streams.huffman_stream(codes, w, 8 * 600_000 + 5, seed=5)
+    return [
+        ("html", dfas.html_tokenizer(), streams.html_bytes(1_500_000, 3), None),
+        ("ccomment", dfas.c_comment(True), streams.c_source(700_001, seed=3, comment_frac=0.4), None),
+        ("ac", dfas.aho_corasick(pats), streams.ac_payload(1_200_000, 4, pats), None),
+        ("rand", dfas.random_dfa(64, 6, seed=3), streams.splitmix_bytes(12, 0, 1_000_001), None),
+        ("huff", hd, hb, 8 * 600_000 + 5),
+        ("div7", dfas.div7(), streams.random_bits(8 * 300_000 + 3, 6), 8 * 300_000 + 3),
+    ]
+
+
+@pytest.mark.parametrize("lookback", [32, 64, 256])
+def test_lookback_window_parity(lookback):
+    for name, d, data, length in _wl_cases():
+        exp = seq.run(d, data, length)
+        for k in (1, 2):
+            for chunk in (64, 2048):
+                got, st = gpu_run(d, data, length, k=k, chunk_bytes=chunk, lookback_len=lookback)
+                assert got == exp, (name, lookback, k, chunk, st)
+                assert st["lookback_len"] == lookback
+
+
+def test_lookback_window_reduces_misses():
+    d = dfas.html_tokenizer()
+    data = streams.html_bytes(4_000_000, 5)
+    _, st1 = gpu_run(d, data, k=2, chunk_bytes=1024)
+    _, st64 = gpu_run(d, data, k=2, chunk_bytes=1024, lookback_len=64)
+    assert st64["reexec_chunks"] < st1["reexec_chunks"] / 4, (st1, st64)
+
+
+@pytest.mark.parametrize("lookback", [0, 64])
+def test_lookback_seqmerge_and_shards(lookback):
+    d = dfas.html_tokenizer()
+    data = streams.html_bytes(2_000_000, 8)
+    exp = seq.run(d, data)
+    got, _ = gpu_run(d, data, k=2, merge=fsmspec.FSM_MERGE_SEQUENTIAL, lookback_len=lookback)
+    assert got == exp
+    buf, base = dev(data)
+    G, L = 3, data.size
+    bounds = [L * g // G // 32 * 32 for g in range(G)] + [L]
+    with FSM.from_dfa(d) as f:
+        f.set_options(lookback_len=lookback)
+        x, total = d.start, 0
+        for g in range(G):
+            lo, hi = bounds[g], bounds[g + 1]
+            m, sh = f.run_shard(base + lo, hi - lo, halo=(base + lo - 1) if g else None,
+                                halo_len=1 if g else 0, k=2, keep=True)
+            for s, e, c in m.slots():
+                assert (e, c) == seq.run_from(d, s, data[lo:hi])
+            hit = [(e, c) for s, e, c in m.slots() if s == x]
+            e, c = hit[0] if hit else f.shard_fixup(sh, x)
+            x, total = e, total + c
+        assert (x, total) == exp

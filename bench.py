@@ -217,6 +217,7 @@ def main():
                     help="skip the sequential-merge ablation run (Fig. 4a, SURVEY 8.a11)")
     args = ap.parse_args()
     w = make_workload(args)
+    w["lookback"] = args.lookback if args.lookback >= 0 else {"c5": 0, "c1": 64, "c4": 64, "c2": 32, "c3": 32}[args.config]
     if args.impl == "reference":
         return run_reference(args, w)
 
@@ -256,8 +257,7 @@ def main():
 
     f = FSM.from_dfa(d)
     f.set_stream(stream.cuda_stream)
-    lookback = args.lookback if args.lookback >= 0 else {"c5": 0, "c1": 64, "c4": 64, "c2": 32, "c3": 32}[args.config]
-    w["lookback"] = lookback
+    lookback = w["lookback"]
     f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback)
     res = torch.zeros(4, dtype=torch.int32, device=dev)
     small = total < 4 * 126_000_000

@@ -17,6 +17,7 @@
 #include "fixup_kernel.cuh"
 #include "host_tables.h"
 #include "seqmerge_kernel.cuh"
+#include "spec_kernel.cuh"
 #include "speck_kernel.cuh"
 
 using namespace speck;
@@ -31,13 +32,15 @@ typedef void (*KernelFn)(Params);
 typedef void (*FixFn)(FixParams);
 typedef void (*SeqLocalFn)(Params, SeqBuf);
 typedef void (*SeqWalkFn)(Params, SeqBuf);
+typedef void (*SpecFn)(Params, uint16_t *);
 
 // Kernel instantiations live in one translation unit per table variant (kernels_*.cu, compiled in
 // parallel); each exports these accessors.
 #define FSM_DECLARE_VARIANT(NAME)                                   \
     KernelFn get_kernel_##NAME(int K);                              \
     FixFn get_fix_##NAME();                                         \
-    void get_seq_##NAME(int K, SeqLocalFn &l, SeqWalkFn &w);
+    void get_seq_##NAME(int K, SeqLocalFn &l, SeqWalkFn &w);       \
+    SpecFn get_spec_##NAME();
 FSM_DECLARE_VARIANT(p4)
 FSM_DECLARE_VARIANT(p8)
 FSM_DECLARE_VARIANT(h8)
@@ -62,6 +65,16 @@ static FixFn get_fix(int var)
     case VAR_H8: return get_fix_h8();
     case VAR_B: return get_fix_b();
     default: return get_fix_g();
+    }
+}
+static SpecFn get_spec(int var)
+{
+    switch (var) {
+    case VAR_P4: return get_spec_p4();
+    case VAR_P8: return get_spec_p8();
+    case VAR_H8: return get_spec_h8();
+    case VAR_B: return get_spec_b();
+    default: return get_spec_g();
     }
 }
 static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
@@ -113,6 +126,9 @@ struct fsm {
     uint8_t *d_stage[2] = {nullptr, nullptr};
     size_t stage_bytes = 0;
     cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
+    // look-back window pre-pass output
+    uint16_t *d_spec = nullptr;
+    size_t spec_cap = 0;
     // sequential-merge ablation buffers
     SeqBuf seq{};
     size_t seq_cap = 0;
@@ -185,6 +201,7 @@ static void free_all(fsm *f)
     cudaFree(f->d_fix);
     cudaFree(f->d_stage[0]);
     cudaFree(f->d_stage[1]);
+    cudaFree(f->d_spec);
     cudaFree(f->seq.S);
     cudaFree(f->seq.E);
     cudaFree(f->seq.C);
@@ -458,6 +475,30 @@ static int launch_run(fsm *f, const RunSpec &r)
 
     const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes)).total;
 
+    if (p.lookback >= 32) {
+        // a3 pre-pass: ranked look-back candidates per chunk (spec_kernel.cuh)
+        const uint64_t nch = len_bytes == 0 ? 1 : (len_bytes + chunk - 1) / chunk;
+        p.spec_stride = (uint32_t)r.k + kExt;
+        const size_t need = nch * p.spec_stride;
+        if (need > f->spec_cap) {
+            cudaStreamSynchronize(f->stream);
+            cudaFree(f->d_spec);
+            f->d_spec = nullptr;
+            f->spec_cap = 0;
+            CK(cudaMalloc(&f->d_spec, need * 2));
+            f->spec_cap = need;
+        }
+        SpecFn sf = get_spec(var);
+        const size_t smem_s = std::max<size_t>(16, scratch_offset(var, p.table_bytes));
+        CK(cudaFuncSetAttribute((const void *)sf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_s));
+        int occ_s = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, sf, kThreads, smem_s));
+        const uint64_t blocks = std::min<uint64_t>((nch + kThreads - 1) / kThreads, (uint64_t)std::max(occ_s, 1) * f->num_sms);
+        sf<<<(uint32_t)blocks, kThreads, smem_s, f->stream>>>(p, f->d_spec);
+        CK(cudaGetLastError());
+        p.spec = f->d_spec;
+    }
+
     if (r.merge == FSM_MERGE_SEQUENTIAL) {
         if (r.keyed) return FSM_EINVAL;
         return launch_seq(f, p, var, K, T);
@@ -495,7 +536,8 @@ static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T)
     const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
     if (nch * K > f->seq_cap) {
         cudaStreamSynchronize(f->stream);
-        cudaFree(f->seq.S);
+        cudaFree(f->d_spec);
+    cudaFree(f->seq.S);
         cudaFree(f->seq.E);
         cudaFree(f->seq.C);
         f->seq = SeqBuf{};

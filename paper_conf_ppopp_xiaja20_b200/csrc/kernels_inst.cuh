@@ -3,6 +3,7 @@
 // kernels through the accessors defined here.  K list = kKs in fsmspec.cu.
 #include "fixup_kernel.cuh"
 #include "seqmerge_kernel.cuh"
+#include "spec_kernel.cuh"
 #include "speck_kernel.cuh"
 
 using namespace speck;
@@ -10,6 +11,7 @@ typedef void (*KernelFn)(Params);
 typedef void (*FixFn)(FixParams);
 typedef void (*SeqLocalFn)(Params, SeqBuf);
 typedef void (*SeqWalkFn)(Params, SeqBuf);
+typedef void (*SpecFn)(Params, uint16_t *);
 
 #define FSM_CAT2(a, b) a##b
 #define FSM_CAT(a, b) FSM_CAT2(a, b)
@@ -43,3 +45,5 @@ void FSM_CAT(get_seq_, FSM_VAR_NAME)(int K, SeqLocalFn &l, SeqWalkFn &w)
     default: l = seq_local_kernel<16, FSM_VAR>; w = seq_walk_kernel<16, FSM_VAR>; break;
     }
 }
+
+SpecFn FSM_CAT(get_spec_, FSM_VAR_NAME)() { return spec_kernel<FSM_VAR>; }

@@ -1,0 +1,90 @@
+// spec_kernel.cuh -- a3 look-back speculation with a window (reading R7), as a pre-pass.
+//
+// For every chunk (start byte b): the image of x[b-Lw-1] (the host look-back table) is run
+// through the Lw bytes x[b-Lw .. b) and the reached states are ranked by multiplicity (how many
+// image states reach each), ties to the smaller id; the top k + kExt distinct states are written
+// to spec[chunk][0 .. k + kExt) (0xFFFF = none).  Chunks whose window would reach before the start
+// of a known-start run get the single exact state; keyed runs and short prefixes fall back to the
+// depth-1 look-back.  One thread per chunk; the fused kernel then only reads its chunk's list.
+// Kept out of the fused kernel so its 16-chain working set does not raise the hot loop's register
+// allocation.
+#pragma once
+#include "speck_kernel.cuh"
+
+namespace speck {
+
+template <int VAR>
+__global__ void __launch_bounds__(kThreads) spec_kernel(Params p, uint16_t *__restrict__ spec)
+{
+    using TB = typename TableFor<VAR>::type;
+    extern __shared__ __align__(16) uint8_t smem[];
+    check_smem_window(VAR, scratch_offset(VAR, p.table_bytes));
+    TB tb;
+    tb.setup(smem, p.table, p.n_states, kconst(p));
+    __syncthreads();
+    const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
+    const uint32_t ksel = p.k, stride = p.spec_stride, Lw = p.lookback;
+    const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
+    for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nch; g += (uint64_t)gridDim.x * blockDim.x) {
+        uint16_t *out = spec + g * stride;
+        const uint64_t b = g * p.chunk;
+        uint32_t written = 0;
+        if (g == 0 && !p.keyed) {
+            out[written++] = (uint16_t)start_state;
+        } else if (b >= Lw + 1 && p.aligned) {
+            const uint32_t c0 = __ldg(p.in + b - Lw - 1);
+            const uint32_t ni = __ldg(p.nimg + c0);
+            uint32_t y[KMAX];
+#pragma unroll
+            for (int i = 0; i < KMAX; i++) y[i] = (uint32_t)__ldg(p.lb + c0 * KMAX + ((uint32_t)i < ni ? i : 0));
+            for (uint32_t o = 0; o < Lw; o += 32) {
+                const Bytes32 x = ldg256(p.in + b - Lw + o);
+#pragma unroll 1
+                for (int t = 0; t < 32; t++) {
+                    const uint32_t byte = (x.w[t >> 2] >> (8 * (t & 3))) & 0xFFu;
+                    const typename TB::Row r = tb.row(byte);
+                    uint32_t dummy = 0;
+#pragma unroll
+                    for (int i = 0; i < KMAX; i++) y[i] = tb.apply(r, y[i], dummy);
+                }
+            }
+            uint32_t mult[KMAX];
+#pragma unroll
+            for (int i = 0; i < KMAX; i++) {
+                uint32_t m = 0;
+#pragma unroll
+                for (int j = 0; j < KMAX; j++) m += ((uint32_t)j < ni && y[j] == y[i]) ? 1u : 0u;
+                mult[i] = (uint32_t)i < ni ? m : 0u;
+            }
+            // selection: repeatedly take the best remaining (multiplicity desc, id asc)
+            for (; written < stride; written++) {
+                uint32_t bm = 0, bs = NOSTATE;
+#pragma unroll
+                for (int i = 0; i < KMAX; i++)
+                    if (mult[i] > bm || (mult[i] == bm && mult[i] && y[i] < bs)) {
+                        bm = mult[i];
+                        bs = y[i];
+                    }
+                if (!bm) break;
+#pragma unroll
+                for (int i = 0; i < KMAX; i++)
+                    if (y[i] == bs) mult[i] = 0;
+                out[written] = (uint16_t)bs;
+            }
+        } else if (!p.keyed && b > 0) {
+            // the window would reach the start of a known-start run: exact state
+            uint32_t st = start_state, dummy = 0;
+            for (uint64_t t = 0; t < b; t++) st = tb.apply(tb.row(__ldg(p.in + t)), st, dummy);
+            out[written++] = (uint16_t)st;
+        } else {
+            const uint32_t c = g == 0 ? p.halo_byte : (uint32_t)__ldg(p.in + b - 1);
+            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), stride);
+            for (; written < ni; written++) out[written] = __ldg(p.lb + c * KMAX + written);
+        }
+        // the first k entries are the speculated set, the rest eager-completion candidates
+        (void)ksel;
+        for (; written < stride; written++) out[written] = 0xFFFFu;
+    }
+}
+
+}  // namespace speck

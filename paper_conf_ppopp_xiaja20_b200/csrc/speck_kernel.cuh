@@ -30,17 +30,17 @@ namespace speck {
 enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
-// in lockstep over the chunk's first 32 bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
+// in lockstep over the chunk's first kExtWindow bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
 constexpr int kExt = 4;
+constexpr uint32_t kExtWindow = 128;  // bytes of lockstep per chunk; |count delta| <= 8 * 128 fits 12 bits
 constexpr uint32_t kExtNone = 0xFFFFu;
 // Threads per tile (one chunk per thread) of the fused kernel, by the number of chains K: large
 // CTAs keep few tiles in flight (short look-back windows) at one CTA per SM; the register budget
 // caps them for large K.
-#ifndef FSM_SMALLK_THREADS
-#define FSM_SMALLK_THREADS 1024
-#endif
-__host__ __device__ constexpr int max_threads(int K) { return K <= 3 ? FSM_SMALLK_THREADS : K <= 6 ? 512 : 256; }
-__host__ __device__ constexpr int min_blocks(int K) { return K <= 3 ? 1024 / FSM_SMALLK_THREADS : 1; }
+// (K = 2, 3 at 768 threads get 85 registers: the multi-chain prologue spills at 64; measured
+// +6 % over 1024 threads for (8, 2, k=2).)
+__host__ __device__ constexpr int max_threads(int K) { return K == 1 ? 1024 : K <= 3 ? 768 : K <= 6 ? 512 : 256; }
+__host__ __device__ constexpr int min_blocks(int) { return 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
 
 // ------------------------------------------------------------------------------- PTX helpers --
@@ -539,64 +539,19 @@ __device__ __forceinline__ void speculate(const TB &tb, const Params &p, uint64_
         return;
     }
     const uint32_t ksel = p.k;
-    const uint32_t Lw = p.lookback;
-    if (!first_chunk && Lw >= 32 && p.aligned && b >= Lw + 1) {
-        const uint32_t c0 = __ldg(p.in + b - Lw - 1);
-        const uint32_t ni = __ldg(p.nimg + c0);
-        uint32_t y[KMAX];
+    if (p.spec) {  // ranked candidates from the look-back pre-pass (spec_kernel.cuh)
+        const uint16_t *c = p.spec + (b / p.chunk) * p.spec_stride;
 #pragma unroll
-        for (int i = 0; i < KMAX; i++) y[i] = (uint32_t)__ldg(p.lb + c0 * KMAX + ((uint32_t)i < ni ? i : 0));
-        for (uint32_t o = 0; o < Lw; o += 32) {
-            const Bytes32 x = ldg256(p.in + b - Lw + o);
-#pragma unroll 1
-            for (int t = 0; t < 32; t++) {
-                const uint32_t byte = (x.w[t >> 2] >> (8 * (t & 3))) & 0xFFu;
-                const typename TB::Row r = tb.row(byte);
-                uint32_t dummy = 0;
-#pragma unroll
-                for (int i = 0; i < KMAX; i++) y[i] = tb.apply(r, y[i], dummy);
+        for (int s = 0; s < K; s++)
+            if ((uint32_t)s < ksel) {
+                const uint32_t v = __ldg(c + s);
+                S[s] = v == 0xFFFFu ? NOSTATE : v;
             }
+#pragma unroll
+        for (int q = 0; q < kExt; q++) {
+            const uint32_t v = __ldg(c + ksel + q);
+            X[q] = v == 0xFFFFu ? NOSTATE : v;
         }
-        // rank the distinct reached states by multiplicity (over the ni real candidates)
-        uint32_t mult[KMAX];
-#pragma unroll
-        for (int i = 0; i < KMAX; i++) {
-            uint32_t m = 0;
-#pragma unroll
-            for (int j2 = 0; j2 < KMAX; j2++) m += ((uint32_t)j2 < ni && y[j2] == y[i]) ? 1u : 0u;
-            mult[i] = (uint32_t)i < ni ? m : 0u;
-        }
-        // selection: repeatedly take the best remaining (mult desc, id asc), then retire it
-#pragma unroll 1
-        for (uint32_t r = 0; r < (uint32_t)(K + kExt); r++) {
-            uint32_t bm = 0, bs = NOSTATE;
-#pragma unroll
-            for (int i = 0; i < KMAX; i++)
-                if (mult[i] > bm || (mult[i] == bm && mult[i] && y[i] < bs)) {
-                    bm = mult[i];
-                    bs = y[i];
-                }
-            if (!bm) break;
-#pragma unroll
-            for (int i = 0; i < KMAX; i++)
-                if (y[i] == bs) mult[i] = 0;
-            if (r < ksel) {
-#pragma unroll
-                for (int s = 0; s < K; s++)
-                    if ((uint32_t)s == r) S[s] = bs;
-            } else {
-#pragma unroll
-                for (int q = 0; q < kExt; q++)
-                    if ((uint32_t)q + ksel == r) X[q] = bs;
-            }
-        }
-        return;
-    }
-    if (!first_chunk && !p.keyed && Lw >= 32 && b < Lw + 1 && b > 0) {
-        // the window reaches the start of the run: run it exactly from the known start
-        uint32_t st = start_state, dummy = 0;
-        for (uint64_t t = 0; t < b; t++) st = tb.apply(tb.row(__ldg(p.in + t)), st, dummy);
-        S[0] = st;
         return;
     }
     const uint32_t c = first_chunk ? p.halo_byte : (uint32_t)__ldg(p.in + b - 1);
@@ -932,23 +887,35 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
                     cu[q] = 0;
                     nlive += live[q];
                 }
+                // window: the stashed first 32 bytes, then up to kExtWindow bytes from global (L2)
+                const uint32_t wlen = (uint32_t)((e - b) < kExtWindow ? (e - b) : kExtWindow) & ~31u;
 #pragma unroll 1
-                for (int pos = 0; pos < 32 && nlive > 0; pos++) {
-                    const uint32_t byte = (st32[pos >> 2] >> (8 * (pos & 3))) & 0xFFu;
-                    const typename TB::Row r = tb.row(byte);
+                for (uint32_t blk = 0; blk < wlen && nlive > 0; blk += 32) {
+                    Bytes32 xb;
+                    if (blk == 0) {
 #pragma unroll
-                    for (int l = 0; l < K; l++) y[l] = tb.apply(r, y[l], cy[l]);
+                        for (int q = 0; q < 8; q++) xb.w[q] = st32[q];
+                    } else {
+                        xb = ldg256(p.in + b + blk);
+                    }
+#pragma unroll 1
+                    for (int pos = 0; pos < 32 && nlive > 0; pos++) {
+                        const uint32_t byte = (xb.w[pos >> 2] >> (8 * (pos & 3))) & 0xFFu;
+                        const typename TB::Row r = tb.row(byte);
 #pragma unroll
-                    for (int q = 0; q < kExt; q++) {
-                        if (!live[q]) continue;
-                        u[q] = tb.apply(r, u[q], cu[q]);
+                        for (int l = 0; l < K; l++) y[l] = tb.apply(r, y[l], cy[l]);
 #pragma unroll
-                        for (int l = 0; l < K; l++)
-                            if (live[q] && S[l] != NOSTATE && y[l] == u[q]) {
-                                live[q] = false;
-                                nlive--;
-                                ent[q] = Xc[q] | ((uint32_t)l << 16) | (((cu[q] - cy[l]) & 0xFFFu) << 20);
-                            }
+                        for (int q = 0; q < kExt; q++) {
+                            if (!live[q]) continue;
+                            u[q] = tb.apply(r, u[q], cu[q]);
+#pragma unroll
+                            for (int l = 0; l < K; l++)
+                                if (live[q] && S[l] != NOSTATE && y[l] == u[q]) {
+                                    live[q] = false;
+                                    nlive--;
+                                    ent[q] = Xc[q] | ((uint32_t)l << 16) | (((cu[q] - cy[l]) & 0xFFFu) << 20);
+                                }
+                        }
                     }
                 }
             }

@@ -58,6 +58,8 @@ struct Params {
     uint32_t ntiles;
     uint32_t k;                    // speculated states in use (<= template K)
     uint32_t lookback;             // look-back window in bytes (0/1: the preceding byte only)
+    const uint16_t *spec;          // window look-back: ranked candidates per chunk (spec_kernel), or null
+    uint32_t spec_stride;          // candidates per chunk in `spec` (k + kExt)
     uint32_t aligned;              // `in` is 32-byte aligned
     const void *table;             // variant image in global memory
     uint32_t n_states;             // internal states (incl. sink)

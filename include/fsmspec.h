@@ -53,7 +53,9 @@ enum {
     FSM_VARIANT_P8 = 1,  /* N <= 8:   packed 8 x u8 row per symbol, lane-replicated smem, PRMT chain */
     FSM_VARIANT_B = 2,   /* N <= 256: u16 entries (next | count << 8) in shared memory            */
     FSM_VARIANT_G = 3,   /* any N:    u32 entries (next | count << 16) in global memory / L2      */
-    FSM_VARIANT_H8 = 4   /* N <= 8 (byte mode): half rows of 4 states, one LDS.32 per chain step   */
+    FSM_VARIANT_H8 = 4,  /* N <= 8 (byte mode): half rows of 4 states, one LDS.32 per chain step   */
+    FSM_VARIANT_HS = 5   /* byte mode, N <= 32768: hot-state row caching (Sec. 4.2): the most frequent
+                            states' rows in shared memory (u16), the rest from the u32 table in L2 */
 };
 
 /* Merge strategies: the paper's parallel merge (default) and its sequential-merge baseline
@@ -101,13 +103,13 @@ int fsm_run_spec_k(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k,
 
 /* Result record written to device memory by the asynchronous call. */
 typedef struct {
-    uint32_t final_state;   /* internal id; == n_states means an out-of-alphabet byte was seen */
+    uint32_t final_state;   /* == n_states means an out-of-alphabet byte was seen */
     uint32_t status;        /* 0 */
     uint64_t accept_count;
 } fsm_result;
 
-/* fsm_run_spec_k_async: as fsm_run_spec_k, but only enqueues the work on the handle's stream and
- * writes an fsm_result to `dev_result` (device pointer, 16-byte aligned).  No host
+/* fsm_run_spec_k_async: as fsm_run_spec_k, but only enqueues the work on the handle's stream; the
+ * kernel writes an fsm_result to `dev_result` (device pointer, 8-byte aligned).  No host
  * synchronisation.  `final_state == n_states` signals FSM_ESYMBOL (when alphabet < 256). */
 int fsm_run_spec_k_async(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k,
                          fsm_result *dev_result);

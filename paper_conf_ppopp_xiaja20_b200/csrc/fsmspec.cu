@@ -46,6 +46,7 @@ FSM_DECLARE_VARIANT(p8)
 FSM_DECLARE_VARIANT(h8)
 FSM_DECLARE_VARIANT(b)
 FSM_DECLARE_VARIANT(g)
+FSM_DECLARE_VARIANT(hs)
 
 static KernelFn get_kernel(int var, int K)
 {
@@ -53,6 +54,7 @@ static KernelFn get_kernel(int var, int K)
     case VAR_P4: return get_kernel_p4(K);
     case VAR_P8: return get_kernel_p8(K);
     case VAR_H8: return get_kernel_h8(K);
+    case VAR_HS: return get_kernel_hs(K);
     case VAR_B: return get_kernel_b(K);
     default: return get_kernel_g(K);
     }
@@ -63,6 +65,7 @@ static FixFn get_fix(int var)
     case VAR_P4: return get_fix_p4();
     case VAR_P8: return get_fix_p8();
     case VAR_H8: return get_fix_h8();
+    case VAR_HS: return get_fix_hs();
     case VAR_B: return get_fix_b();
     default: return get_fix_g();
     }
@@ -73,6 +76,7 @@ static SpecFn get_spec(int var)
     case VAR_P4: return get_spec_p4();
     case VAR_P8: return get_spec_p8();
     case VAR_H8: return get_spec_h8();
+    case VAR_HS: return get_spec_hs();
     case VAR_B: return get_spec_b();
     default: return get_spec_g();
     }
@@ -83,6 +87,7 @@ static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
     case VAR_P4: get_seq_p4(K, l, w); break;
     case VAR_P8: get_seq_p8(K, l, w); break;
     case VAR_H8: get_seq_h8(K, l, w); break;
+    case VAR_HS: get_seq_hs(K, l, w); break;
     case VAR_B: get_seq_b(K, l, w); break;
     default: get_seq_g(K, l, w); break;
     }
@@ -106,8 +111,14 @@ struct fsm {
     int auto_variant = VAR_G;
     fsm_options opt{};
     // device tables
-    void *d_img[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
-    uint32_t img_bytes[5] = {0, 0, 0, 0, 0};
+    void *d_img[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    uint32_t img_bytes[6] = {0, 0, 0, 0, 0, 0};
+    // static-frequency renumbering (hot-state caching): user <-> internal ids
+    bool renumbered = false;
+    std::vector<uint32_t> perm, inv;
+    uint32_t *d_inv = nullptr;
+    uint32_t hot_rows = 0;
+    uint32_t start_int = 0;
     uint16_t *d_lb = nullptr;
     uint8_t *d_nimg = nullptr;
     uint32_t *d_bittab = nullptr;
@@ -190,7 +201,8 @@ extern "C" int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint
 
 static void free_all(fsm *f)
 {
-    for (int i = 0; i < 5; i++) cudaFree(f->d_img[i]);
+    for (int i = 0; i < 6; i++) cudaFree(f->d_img[i]);
+    cudaFree(f->d_inv);
     cudaFree(f->d_lb);
     cudaFree(f->d_nimg);
     cudaFree(f->d_bittab);
@@ -251,11 +263,22 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
     f->start = start;
     f->mode = input_mode;
     build_byte_dfa(table, n_states, alphabet, accept_mask, bits, f->dfa);
+    f->start_int = start;
+    if (!bits && f->dfa.n > 256 && f->dfa.n <= 32768) {
+        // tables beyond shared memory: hot-state caching needs hot rows = small ids (Sec. 4.2)
+        renumber_by_frequency(f->dfa, n_states, f->perm, f->inv);
+        f->renumbered = true;
+        f->start_int = f->perm[start];
+    }
     f->lb.resize(256 * KMAX);
     f->nimg.resize(256);
     build_lookback(f->dfa, f->lb.data(), f->nimg.data());
     const uint32_t n = f->dfa.n;
-    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B : VAR_G;
+    // N > 256: the u32 table in L2 with the L1 acting as a hardware hot-row cache (G) measured faster
+    // up to ~2K states (1027-state AC: 1.12 vs 0.98 TB/s); beyond that explicit hot-state caching in
+    // shared memory wins (4121-state AC: 0.90 vs 0.76 TB/s).  Both use the frequency renumbering.
+    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B
+                    : (f->renumbered && n > 2048) ? VAR_HS : VAR_G;
     f->opt.chunk_bytes = 0;
     f->opt.threads_per_tile = 0;  // auto: max_threads(K)
     f->opt.variant = FSM_VARIANT_AUTO;
@@ -294,6 +317,14 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         if ((rc = upload(&f->d_img[VAR_G], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_G] = 0;
     }
+    if (!bits && f->dfa.n <= 32768) {
+        // hot rows: as many u16 rows (512 B each) as fit next to the kernel's scratch
+        f->hot_rows = std::min<uint32_t>(f->dfa.n, 384);
+        auto img = image_hs(f->dfa, f->hot_rows);
+        if ((rc = upload(&f->d_img[VAR_HS], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_HS] = (uint32_t)img.size();
+    }
+    if (f->renumbered && (rc = upload(&f->d_inv, f->inv.data(), f->inv.size() * 4))) return fail(rc);
     if ((rc = upload(&f->d_lb, f->lb.data(), f->lb.size() * 2))) return fail(rc);
     if ((rc = upload(&f->d_nimg, f->nimg.data(), f->nimg.size()))) return fail(rc);
     if (bits && (rc = upload(&f->d_bittab, f->dfa.bittab.data(), f->dfa.bittab.size() * 4))) return fail(rc);
@@ -342,7 +373,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
-    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_H8) return FSM_EINVAL;
+    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_HS) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
@@ -371,6 +402,7 @@ extern "C" int fsm_get_stats(const fsm_t *f, fsm_stats *s)
 
 // ----------------------------------------------------------------------------------- runs ----
 struct RunSpec {
+    uint32_t *user_out;    // async API: user-visible result written by the kernel (may be null)
     const uint8_t *in;
     uint64_t len_sym;      // symbols
     uint32_t k;
@@ -472,7 +504,19 @@ static int launch_run(fsm *f, const RunSpec &r)
     p.k_512 = 512;
     p.k_1e27 = 1u << 27;
     p.k_2 = 2;
+    p.table_g = static_cast<const uint32_t *>(f->d_img[VAR_G]);
+    p.hot_rows = f->hot_rows;
+    p.inv = f->d_inv;
+    p.user_out = r.user_out;
 
+    if (var == VAR_HS) {
+        // as many hot rows as fit next to this launch's scratch (227 KB per CTA)
+        const uint32_t scratch = Layout(T, K, 0).total;
+        const uint32_t avail = scratch < 232448u ? 232448u - scratch : 0u;
+        const uint32_t hot = std::min<uint32_t>(f->hot_rows, avail / 512);
+        p.hot_rows = hot;
+        p.table_bytes = hot * 512;
+    }
     const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes)).total;
 
     if (p.lookback >= 32) {
@@ -595,16 +639,17 @@ static int finish_sync(fsm *f, const DevResult *dres)
 }
 
 static bool is_sink(const fsm *f, uint32_t s) { return f->dfa.sink != 0xFFFFFFFFu && s == f->dfa.sink; }
+static uint32_t to_user(const fsm *f, uint32_t s) { return f->renumbered && s < f->inv.size() ? f->inv[s] : s; }
+static uint32_t to_int(const fsm *f, uint32_t s) { return f->renumbered && s < f->perm.size() ? f->perm[s] : s; }
 
 extern "C" int fsm_run_spec_k_async(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k, fsm_result *dev_result)
 {
     int rc = check_run_args(f, input, len, k);
     if (rc) return rc;
     if (!dev_result) return FSM_EINVAL;
-    RunSpec r{input, len, k, false, 0, f->start, nullptr, f->d_result, -1, f->opt.merge};
-    if ((rc = launch_run(f, r))) return rc;
-    CK(cudaMemcpyAsync(dev_result, f->d_result, sizeof(fsm_result), cudaMemcpyDeviceToDevice, f->stream));
-    return FSM_OK;
+    RunSpec r{reinterpret_cast<uint32_t *>(dev_result), input, len, k, false, 0, f->start_int, nullptr, f->d_result,
+              -1, f->opt.merge};
+    return launch_run(f, r);  // the last tile writes the user-visible result into dev_result
 }
 
 extern "C" int fsm_run_spec_k(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k, uint32_t *final_state,
@@ -613,11 +658,11 @@ extern "C" int fsm_run_spec_k(fsm_t *f, const uint8_t *input, uint64_t len, uint
     int rc = check_run_args(f, input, len, k);
     if (rc) return rc;
     if (!final_state || !accept_count) return FSM_EINVAL;
-    RunSpec r{input, len, k, false, 0, f->start, nullptr, f->d_result, -1, f->opt.merge};
+    RunSpec r{nullptr, input, len, k, false, 0, f->start_int, nullptr, f->d_result, -1, f->opt.merge};
     if ((rc = launch_run(f, r))) return rc;
     if ((rc = finish_sync(f, f->d_result))) return rc;
     if (is_sink(f, f->h_result->final_state)) return FSM_ESYMBOL;
-    *final_state = f->h_result->final_state;
+    *final_state = to_user(f, f->h_result->final_state);
     *accept_count = f->h_result->count;
     return FSM_OK;
 }
@@ -659,7 +704,7 @@ extern "C" int fsm_run_spec_k_host(fsm_t *f, const uint8_t *host_input, uint64_t
         // chain: piece pi starts from piece pi-1's result (d_result[0]); it writes to d_result[pi&1 ^ ...]
         DevResult *res = f->d_result + ((pi + 1) & 1);
         const DevResult *prev = pi == 0 ? nullptr : f->d_result + (pi & 1);
-        RunSpec r{f->d_stage[sb], sym, k, false, 0, f->start, prev, res, -1, FSM_MERGE_PARALLEL};
+        RunSpec r{nullptr, f->d_stage[sb], sym, k, false, 0, f->start_int, prev, res, -1, FSM_MERGE_PARALLEL};
         if ((rc = launch_run(f, r))) return rc;
         CK(cudaEventRecord(f->ev_used[sb], f->stream));
         chunks += f->last.chunks;
@@ -670,7 +715,7 @@ extern "C" int fsm_run_spec_k_host(fsm_t *f, const uint8_t *host_input, uint64_t
     f->last.chunks = chunks;
     f->last.tiles = tiles;
     if (is_sink(f, f->h_result->final_state)) return FSM_ESYMBOL;
-    *final_state = f->h_result->final_state;
+    *final_state = to_user(f, f->h_result->final_state);
     *accept_count = f->h_result->count;
     return FSM_OK;
 }
@@ -690,7 +735,7 @@ extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const
         CK(cudaStreamSynchronize(f->stream));
         hb = h;
     }
-    RunSpec r{input, len, k, keyed, hb, f->start, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL};
+    RunSpec r{nullptr, input, len, k, keyed, hb, f->start_int, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL};
     if ((rc = launch_run(f, r))) return rc;
     if ((rc = finish_sync(f, f->d_result))) return rc;
     const DevResult *hr = f->h_result;
@@ -699,13 +744,14 @@ extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const
     if (!keyed) {
         m.valid_mask = 1;
         m.start[0] = f->start;
-        m.end[0] = hr->final_state;
+        m.end[0] = to_user(f, hr->final_state);
         m.count[0] = hr->count;
     } else {
         m.valid_mask = hr->valid_mask & ((1u << KMAX) - 1);
         for (int s = 0; s < KMAX; s++) {
-            m.start[s] = hr->start[s];
-            m.end[s] = hr->end[s];
+            const bool v = (m.valid_mask >> s) & 1u;
+            m.start[s] = v ? to_user(f, hr->start[s]) : hr->start[s];
+            m.end[s] = v ? to_user(f, hr->end[s]) : hr->end[s];
             m.count[s] = hr->mcount[s];
         }
     }
@@ -724,7 +770,7 @@ extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const
 
 extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, uint32_t *end, uint64_t *count)
 {
-    if (!f || !st || !end || !count || true_start >= f->dfa.n) return FSM_EINVAL;
+    if (!f || !st || !end || !count || true_start >= f->n_user) return FSM_EINVAL;
     for (int s = 0; s < KMAX; s++)
         if (((st->map.valid_mask >> s) & 1u) && st->map.start[s] == true_start) {
             *end = st->map.end[s];
@@ -740,16 +786,17 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
     fp.limit = (uint64_t)1 << 20;
     fp.table = f->d_img[var];
     fp.n_states = f->dfa.n;
-    fp.x = true_start;
+    fp.x = to_int(f, true_start);
     fp.k = st->map.k;
     fp.valid_mask = st->map.valid_mask;
     for (int s = 0; s < KMAX; s++) {
-        fp.start[s] = st->map.start[s];
-        fp.end[s] = st->map.end[s];
+        const bool v = (st->map.valid_mask >> s) & 1u;
+        fp.start[s] = v ? to_int(f, st->map.start[s]) : st->map.start[s];
+        fp.end[s] = v ? to_int(f, st->map.end[s]) : st->map.end[s];
         fp.count[s] = st->map.count[s];
     }
     fp.out = f->d_fix;
-    fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2};
+    fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows};
     FixFn fn = get_fix(var);
     const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -759,16 +806,17 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
     CK(cudaMemcpyAsync(h, f->d_fix, sizeof(h), cudaMemcpyDeviceToHost, f->stream));
     CK(cudaStreamSynchronize(f->stream));
     if (h[0]) {
-        *end = (uint32_t)h[1];
+        *end = to_user(f, (uint32_t)h[1]);
         *count = h[2];
         return FSM_OK;
     }
     // no convergence: exact parallel re-run of the shard from the true start
-    RunSpec r{st->input, st->len, st->k, false, 0, true_start, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL};
+    RunSpec r{nullptr, st->input, st->len, st->k, false, 0, to_int(f, true_start), nullptr, f->d_result, -1,
+              FSM_MERGE_PARALLEL};
     int rc = launch_run(f, r);
     if (rc) return rc;
     if ((rc = finish_sync(f, f->d_result))) return rc;
-    *end = f->h_result->final_state;
+    *end = to_user(f, f->h_result->final_state);
     *count = f->h_result->count;
     return FSM_OK;
 }

@@ -63,6 +63,47 @@ inline int build_byte_dfa(const uint32_t *table, uint32_t n_states, uint32_t alp
     return 0;
 }
 
+// Static-frequency renumbering for hot-state caching (Sec. 4.2): the frequency of a state is its
+// in-degree in the transition table ("the frequency of each of states a and c is 4");
+// states are renumbered by decreasing frequency (ties: smaller id first) so that the hottest rows
+// are the ids [0, H).  The sink (if any) keeps the last id.  perm[old] = new, inv[new] = old.
+inline void renumber_by_frequency(ByteDFA &d, uint32_t n_user, std::vector<uint32_t> &perm,
+                                  std::vector<uint32_t> &inv)
+{
+    std::vector<uint64_t> indeg(d.n, 0);
+    for (uint32_t s = 0; s < n_user; s++)
+        for (uint32_t c = 0; c < 256; c++) indeg[d.next[(size_t)s * 256 + c]]++;
+    std::vector<uint32_t> order(n_user);
+    for (uint32_t s = 0; s < n_user; s++) order[s] = s;
+    std::stable_sort(order.begin(), order.end(),
+                     [&](uint32_t a, uint32_t b) { return indeg[a] != indeg[b] ? indeg[a] > indeg[b] : a < b; });
+    perm.assign(d.n, 0);
+    inv.assign(d.n, 0);
+    for (uint32_t r = 0; r < n_user; r++) {
+        perm[order[r]] = r;
+        inv[r] = order[r];
+    }
+    for (uint32_t s = n_user; s < d.n; s++) perm[s] = inv[s] = s;  // the sink
+    std::vector<uint32_t> nx(d.next.size());
+    std::vector<uint8_t> ic(d.inc.size());
+    for (uint32_t s = 0; s < d.n; s++)
+        for (uint32_t c = 0; c < 256; c++) {
+            nx[(size_t)perm[s] * 256 + c] = perm[d.next[(size_t)s * 256 + c]];
+            ic[(size_t)perm[s] * 256 + c] = d.inc[(size_t)s * 256 + c];
+        }
+    d.next.swap(nx);
+    d.inc.swap(ic);
+}
+
+// HS image: the first `hot` rows as u16 entries next | count << 15 (byte mode, N <= 32768).
+inline std::vector<uint8_t> image_hs(const ByteDFA &d, uint32_t hot)
+{
+    std::vector<uint8_t> img((size_t)hot * 512);
+    uint16_t *p = reinterpret_cast<uint16_t *>(img.data());
+    for (size_t i = 0; i < (size_t)hot * 256; i++) p[i] = (uint16_t)(d.next[i] | ((uint32_t)d.inc[i] << 15));
+    return img;
+}
+
 // Look-back table (reading A5): image of each byte ranked by preimage count, ties -> smaller id.
 // The internal sink is not a source: it is only ever entered through an out-of-alphabet byte,
 // whose image is then exactly {sink}.

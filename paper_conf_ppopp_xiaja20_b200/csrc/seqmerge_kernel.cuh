@@ -148,6 +148,12 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
         p.result->final_state = x;
         p.result->status = 0;
         p.result->count = total;
+        if (p.user_out) {
+            p.user_out[0] = p.inv ? __ldg(p.inv + x) : x;
+            p.user_out[1] = 0;
+            p.user_out[2] = (uint32_t)total;
+            p.user_out[3] = (uint32_t)(total >> 32);
+        }
         atomicAdd(&p.stats->reexec_chunks, reexec);
         atomicAdd(&p.stats->reexec_bytes, rebytes);
     }

@@ -27,7 +27,7 @@
 
 namespace speck {
 
-enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4 };
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
 // in lockstep over the chunk's first kExtWindow bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
@@ -170,8 +170,13 @@ __device__ __forceinline__ void check_smem_window(int var, uint32_t need)
 
 struct KConst {
     uint32_t k_1e24, k_16, k_512, k_1e27, k_2;
+    const uint32_t *gtab;  // full u32 table in global memory (HS variant)
+    uint32_t hot_rows;     // HS: states [0, hot_rows) have their rows in shared memory
 };
-__device__ __forceinline__ KConst kconst(const Params &p) { return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2}; }
+__device__ __forceinline__ KConst kconst(const Params &p)
+{
+    return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2, p.table_g, p.hot_rows};
+}
 
 // ------------------------------------------------------------------- table-placement variants --
 // Every variant exposes
@@ -383,12 +388,59 @@ struct TableG {
     }
 };
 
+// HS: hot-state row caching (Sec. 4.2) for tables that exceed shared
+// memory.  States are renumbered at create time by static frequency -- the in-degree in the
+// transition table, the paper's scheme -- so the hottest states are ids [0, H).  Their rows
+// live in shared memory as u16 entries (next | count << 15, 512 B per row, H up to ~400); the
+// other rows are read from the full u32 table in global memory (L2-resident).  The renumbering
+// replaces the paper's Hot_States[hash(state)] lookup by one compare.
+struct TableHS {
+    const uint8_t *sm;
+    const uint32_t *gt;
+    uint32_t hot;
+    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t, const KConst &kc)
+    {
+        sm = s;
+        gt = kc.gtab;
+        hot = kc.hot_rows;
+        const uint4 *src = static_cast<const uint4 *>(g);
+        uint4 *dst = reinterpret_cast<uint4 *>(s);
+        for (uint32_t i = threadIdx.x; i < hot * 32; i += blockDim.x) dst[i] = __ldg(src + i);
+    }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
+    __device__ __forceinline__ uint32_t lookup(uint32_t st, uint32_t c, uint32_t &cnt) const
+    {
+        if (st < hot) {
+            const uint32_t e = *reinterpret_cast<const uint16_t *>(sm + (st << 9) + (c << 1));
+            cnt += e >> 15;
+            return e & 0x7FFFu;
+        }
+        const uint32_t e = __ldg(gt + ((st << 8) | c));
+        cnt += e >> 16;
+        return e & 0xFFFFu;
+    }
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
+    {
+        const uint32_t c = (w >> (8 * j)) & 0xFFu;
+#pragma unroll
+        for (int s = 0; s < K; s++) cur[s] = lookup(cur[s], c, accf[s]);
+    }
+    using Row = uint32_t;
+    __device__ __forceinline__ Row row(uint32_t c) const { return c; }
+    __device__ __forceinline__ uint32_t apply(Row c, uint32_t st, uint32_t &cnt) const { return lookup(st, c, cnt); }
+};
+
 template <int VAR> struct TableFor;
 template <> struct TableFor<VAR_P4> { using type = TablePacked<VAR_P4>; };
 template <> struct TableFor<VAR_P8> { using type = TablePacked<VAR_P8>; };
 template <> struct TableFor<VAR_B> { using type = TableB; };
 template <> struct TableFor<VAR_G> { using type = TableG; };
 template <> struct TableFor<VAR_H8> { using type = TableH8; };
+template <> struct TableFor<VAR_HS> { using type = TableHS; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <int K, class TB>
@@ -1202,9 +1254,15 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
             DevResult *R = p.result;
             if (!p.keyed) {
                 if (lane == 0) {
-                    R->final_state = x;
+                    R->final_state = x;  // internal id (chains pieces on the device)
                     R->status = 0;
                     R->count = cc;
+                    if (p.user_out) {
+                        p.user_out[0] = p.inv ? __ldg(p.inv + x) : x;
+                        p.user_out[1] = 0;
+                        p.user_out[2] = (uint32_t)cc;
+                        p.user_out[3] = (uint32_t)(cc >> 32);
+                    }
                 }
             } else {
                 const uint32_t c = p.halo_byte;

@@ -83,6 +83,10 @@ struct Params {
     // constants passed at run time so that ptxas cannot strength-reduce the FMA-pipe IMADs into
     // ALU-pipe shifts (the hot loop balances the two pipes): 1 << 24, 16, 512
     uint32_t k_1e24, k_16, k_512, k_1e27, k_2;
+    const uint32_t *table_g;       // full u32 table (HS variant's cold rows)
+    uint32_t hot_rows;             // HS variant: rows cached in shared memory
+    const uint32_t *inv;           // internal -> user state ids (renumbered handles), or null
+    uint32_t *user_out;            // optional: the last tile also writes {user state, 0, count lo, hi} here
 };
 
 }  // namespace speck

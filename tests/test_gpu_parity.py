@@ -35,17 +35,17 @@ def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
     return res, st
 
 
-VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4, "HS": 5}
 
 
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
     return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "H8": n <= 8 and not dfa.bit_mode,
-            "B": n <= 256, "G": True}[var]
+            "B": n <= 256, "G": True, "HS": not dfa.bit_mode and n <= 32768}[var]
 
 
 # --------------------------------------------------------------------- worked example on GPU
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS"])
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
 def test_fig1_worked_example(var, k):
     d = dfas.c_comment(True)
@@ -55,7 +55,7 @@ def test_fig1_worked_example(var, k):
 
 
 # --------------------------------------------------------------------- C1-shaped text
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS"])
 @pytest.mark.parametrize("chunk", [0, 64, 96, 4096])
 def test_c_comment_text(var, chunk):
     d = dfas.c_comment(True)
@@ -156,8 +156,22 @@ def test_aho_corasick():
         data[pos:pos + len(p)] = np.frombuffer(p, np.uint8)
     exp = seq.run(d, data)
     for k in (1, 2, 4):
-        got, _ = gpu_run(d, data, k=k)
-        assert got == exp
+        for var in ("HS", "G"):
+            got, _ = gpu_run(d, data, k=k, variant=VARIANTS[var])
+            assert got == exp, (k, var)
+    # renumbered handle (hot-state caching): the async result is in user state ids
+    with FSM.from_dfa(d) as f:
+        buf, ptr = dev(data)
+        res = torch.zeros(4, dtype=torch.int32, device="cuda")
+        f.run_spec_k_async(ptr, data.size, 2, res.data_ptr())
+        r = res.cpu().numpy().view(np.uint32)
+        assert (int(r[0]), int(r[2]) | (int(r[3]) << 32)) == exp
+        m, sh = f.run_shard(ptr + 1000 * 32, data.size - 1000 * 32, halo=ptr + 1000 * 32 - 1, halo_len=1, k=2,
+                            keep=True)
+        for s_, e_, c_ in m.slots():
+            assert (e_, c_) == seq.run_from(d, s_, data[1000 * 32:])
+        q = int(seq.run(d, data[:1000 * 32])[0])
+        assert f.shard_fixup(sh, q) == seq.run_from(d, q, data[1000 * 32:])
 
 
 # --------------------------------------------------------------------- other entry points

@@ -47,6 +47,7 @@ FSM_DECLARE_VARIANT(h8)
 FSM_DECLARE_VARIANT(b)
 FSM_DECLARE_VARIANT(g)
 FSM_DECLARE_VARIANT(hs)
+FSM_DECLARE_VARIANT(cl)
 
 static KernelFn get_kernel(int var, int K)
 {
@@ -55,6 +56,7 @@ static KernelFn get_kernel(int var, int K)
     case VAR_P8: return get_kernel_p8(K);
     case VAR_H8: return get_kernel_h8(K);
     case VAR_HS: return get_kernel_hs(K);
+    case VAR_CL: return get_kernel_cl(K);
     case VAR_B: return get_kernel_b(K);
     default: return get_kernel_g(K);
     }
@@ -66,6 +68,7 @@ static FixFn get_fix(int var)
     case VAR_P8: return get_fix_p8();
     case VAR_H8: return get_fix_h8();
     case VAR_HS: return get_fix_hs();
+    case VAR_CL: return get_fix_cl();
     case VAR_B: return get_fix_b();
     default: return get_fix_g();
     }
@@ -77,6 +80,7 @@ static SpecFn get_spec(int var)
     case VAR_P8: return get_spec_p8();
     case VAR_H8: return get_spec_h8();
     case VAR_HS: return get_spec_hs();
+    case VAR_CL: return get_spec_cl();
     case VAR_B: return get_spec_b();
     default: return get_spec_g();
     }
@@ -88,6 +92,7 @@ static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
     case VAR_P8: get_seq_p8(K, l, w); break;
     case VAR_H8: get_seq_h8(K, l, w); break;
     case VAR_HS: get_seq_hs(K, l, w); break;
+    case VAR_CL: get_seq_cl(K, l, w); break;
     case VAR_B: get_seq_b(K, l, w); break;
     default: get_seq_g(K, l, w); break;
     }
@@ -111,8 +116,9 @@ struct fsm {
     int auto_variant = VAR_G;
     fsm_options opt{};
     // device tables
-    void *d_img[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
-    uint32_t img_bytes[6] = {0, 0, 0, 0, 0, 0};
+    void *d_img[7] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    uint32_t img_bytes[7] = {0, 0, 0, 0, 0, 0, 0};
+    uint32_t ncls = 0, cl_magic = 0;  // CL variant
     // static-frequency renumbering (hot-state caching): user <-> internal ids
     bool renumbered = false;
     std::vector<uint32_t> perm, inv;
@@ -201,7 +207,7 @@ extern "C" int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint
 
 static void free_all(fsm *f)
 {
-    for (int i = 0; i < 6; i++) cudaFree(f->d_img[i]);
+    for (int i = 0; i < 7; i++) cudaFree(f->d_img[i]);
     cudaFree(f->d_inv);
     cudaFree(f->d_lb);
     cudaFree(f->d_nimg);
@@ -324,6 +330,19 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         if ((rc = upload(&f->d_img[VAR_HS], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_HS] = (uint32_t)img.size();
     }
+    {
+        // CL: byte classes + lane-replicated class-compressed table when it fits shared memory
+        std::vector<uint32_t> cls, rep;
+        const uint32_t nc = cl_pad(byte_classes(f->dfa, cls, rep));
+        if (nc >= 2 && (uint64_t)f->dfa.n * nc <= 1024) {
+            auto img = image_cl(f->dfa, cls, rep);
+            if ((rc = upload(&f->d_img[VAR_CL], img.data(), img.size()))) return fail(rc);
+            f->img_bytes[VAR_CL] = (uint32_t)((256 + (size_t)f->dfa.n * nc) * 128);
+            f->ncls = nc;
+            f->cl_magic = (uint32_t)((((uint64_t)1 << 32) + nc - 1) / nc);
+            if (f->auto_variant == VAR_B) f->auto_variant = VAR_CL;
+        }
+    }
     if (f->renumbered && (rc = upload(&f->d_inv, f->inv.data(), f->inv.size() * 4))) return fail(rc);
     if ((rc = upload(&f->d_lb, f->lb.data(), f->lb.size() * 2))) return fail(rc);
     if ((rc = upload(&f->d_nimg, f->nimg.data(), f->nimg.size()))) return fail(rc);
@@ -373,7 +392,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
-    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_HS) return FSM_EINVAL;
+    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_CL) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
@@ -508,6 +527,8 @@ static int launch_run(fsm *f, const RunSpec &r)
     p.hot_rows = f->hot_rows;
     p.inv = f->d_inv;
     p.user_out = r.user_out;
+    p.ncls = f->ncls;
+    p.cl_magic = f->cl_magic;
 
     if (var == VAR_HS) {
         // as many hot rows as fit next to this launch's scratch (227 KB per CTA)
@@ -796,7 +817,8 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         fp.count[s] = st->map.count[s];
     }
     fp.out = f->d_fix;
-    fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows};
+    fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows,
+                   f->ncls, f->cl_magic};
     FixFn fn = get_fix(var);
     const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

@@ -104,6 +104,49 @@ inline std::vector<uint8_t> image_hs(const ByteDFA &d, uint32_t hot)
     return img;
 }
 
+// Byte classes: bytes whose columns are identical (same next state and count for every state).
+inline uint32_t byte_classes(const ByteDFA &d, std::vector<uint32_t> &cls, std::vector<uint32_t> &rep)
+{
+    cls.assign(256, 0);
+    rep.clear();
+    for (uint32_t c = 0; c < 256; c++) {
+        uint32_t found = 0xFFFFFFFFu;
+        for (uint32_t k = 0; k < rep.size() && found == 0xFFFFFFFFu; k++) {
+            const uint32_t r = rep[k];
+            bool same = true;
+            for (uint32_t s = 0; s < d.n && same; s++)
+                same = d.next[(size_t)s * 256 + c] == d.next[(size_t)s * 256 + r] &&
+                       d.inc[(size_t)s * 256 + c] == d.inc[(size_t)s * 256 + r];
+            if (same) found = k;
+        }
+        if (found == 0xFFFFFFFFu) {
+            found = (uint32_t)rep.size();
+            rep.push_back(c);
+        }
+        cls[c] = found;
+    }
+    return (uint32_t)rep.size();
+}
+
+// CL image: u32 [256] class id per byte, then u32 [N][ncls_pad] entries next * (ncls_pad * 128) | count;
+// ncls_pad = ncls rounded up to even so that the stride is a multiple of 256 and the entry's low
+// byte holds only the count (the kernel adds it with one DP4A).
+inline uint32_t cl_pad(uint32_t ncls) { return (ncls + 1) & ~1u; }
+inline std::vector<uint8_t> image_cl(const ByteDFA &d, const std::vector<uint32_t> &cls,
+                                     const std::vector<uint32_t> &rep)
+{
+    const uint32_t ncls = cl_pad((uint32_t)rep.size()), stride = ncls * 128;
+    std::vector<uint8_t> img((256 + (size_t)d.n * ncls) * 4);
+    uint32_t *p = reinterpret_cast<uint32_t *>(img.data());
+    for (uint32_t c = 0; c < 256; c++) p[c] = cls[c];
+    for (uint32_t s = 0; s < d.n; s++)
+        for (uint32_t k = 0; k < ncls; k++) {
+            const uint32_t r = rep[k < rep.size() ? k : 0];  // padding class: never indexed
+            p[256 + (size_t)s * ncls + k] = d.next[(size_t)s * 256 + r] * stride | d.inc[(size_t)s * 256 + r];
+        }
+    return img;
+}
+
 // Look-back table (reading A5): image of each byte ranked by preimage count, ties -> smaller id.
 // The internal sink is not a source: it is only ever entered through an out-of-alphabet byte,
 // whose image is then exactly {sink}.

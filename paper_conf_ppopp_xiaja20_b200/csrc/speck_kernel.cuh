@@ -27,7 +27,7 @@
 
 namespace speck {
 
-enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5 };
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5, VAR_CL = 6 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
 // in lockstep over the chunk's first kExtWindow bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
@@ -172,10 +172,11 @@ struct KConst {
     uint32_t k_1e24, k_16, k_512, k_1e27, k_2;
     const uint32_t *gtab;  // full u32 table in global memory (HS variant)
     uint32_t hot_rows;     // HS: states [0, hot_rows) have their rows in shared memory
+    uint32_t ncls, cl_magic;  // CL: byte classes, ceil(2^32 / ncls)
 };
 __device__ __forceinline__ KConst kconst(const Params &p)
 {
-    return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2, p.table_g, p.hot_rows};
+    return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2, p.table_g, p.hot_rows, p.ncls, p.cl_magic};
 }
 
 // ------------------------------------------------------------------- table-placement variants --
@@ -434,6 +435,63 @@ struct TableHS {
     __device__ __forceinline__ uint32_t apply(Row c, uint32_t st, uint32_t &cnt) const { return lookup(st, c, cnt); }
 };
 
+// CL: byte-class compressed, lane-replicated table (DFAs with few distinct byte columns, e.g. the
+// HTML tokenizer: 38 states x 24 classes).  Class map: u32 [256][32 lanes] = shared address of the
+// lane's copy of the class row; table: u32 [N][ncls][32 lanes], entry = next * stride | count
+// (stride = ncls * 128, count in bits 0-3).  Every lookup is conflict-free (each lane reads its own
+// bank), the class lookup depends only on the input byte (off the chain), and the chain step is
+// LOP3 + IADD + LDS.32 with the count taken by one DP4A of the entry's low byte.  Chains carry the
+// entry itself (next * stride | count); ids are recovered by a multiply-high.
+struct TableCL {
+    uint32_t cmbase;  // shared address of this lane's class-map column
+    uint32_t stride, magic;
+    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n, const KConst &kc)
+    {
+        const uint32_t base = (uint32_t)__cvta_generic_to_shared(s);
+        const uint32_t ncls = kc.ncls;
+        stride = ncls * 128u;
+        magic = kc.cl_magic;
+        const uint32_t lane = threadIdx.x & 31;
+        cmbase = base + lane * 4;
+        const uint32_t tbase = base + 256 * 128;
+        const uint32_t *img = static_cast<const uint32_t *>(g);
+        for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
+            const uint32_t c = i >> 5, l = i & 31;
+            const uint32_t v = tbase + __ldg(img + c) * 128u + l * 4u;  // image: class id per byte
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(base + c * 128 + l * 4), "r"(v));
+        }
+        for (uint32_t i = threadIdx.x; i < n * ncls * 32; i += blockDim.x) {
+            const uint32_t e = i >> 5, l = i & 31;
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(tbase + e * 128 + l * 4), "r"(__ldg(img + 256 + e)));
+        }
+    }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st * stride; }
+    __device__ __forceinline__ uint32_t id_of(uint32_t cur) const { return __umulhi((cur & ~0xFu) >> 7, magic); }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return id_of(cur); }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
+    {
+        const uint32_t c = (w >> (8 * j)) & 0xFFu;
+        const uint32_t cm = lds_u32(cmbase + (c << 7));  // class row of this lane (off the chain)
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            const uint32_t e = lds_u32((cur[s] & ~0xFu) + cm);
+            acc[s] = dp4a_u(e, 1u, acc[s]);
+            cur[s] = e;
+        }
+    }
+    using Row = uint32_t;
+    __device__ __forceinline__ Row row(uint32_t c) const { return lds_u32(cmbase + (c << 7)); }
+    __device__ __forceinline__ uint32_t apply(Row cm, uint32_t st, uint32_t &cnt) const
+    {
+        const uint32_t e = lds_u32(st * stride + cm);
+        cnt += e & 0xFu;
+        return id_of(e);
+    }
+};
+
 template <int VAR> struct TableFor;
 template <> struct TableFor<VAR_P4> { using type = TablePacked<VAR_P4>; };
 template <> struct TableFor<VAR_P8> { using type = TablePacked<VAR_P8>; };
@@ -441,6 +499,7 @@ template <> struct TableFor<VAR_B> { using type = TableB; };
 template <> struct TableFor<VAR_G> { using type = TableG; };
 template <> struct TableFor<VAR_H8> { using type = TableH8; };
 template <> struct TableFor<VAR_HS> { using type = TableHS; };
+template <> struct TableFor<VAR_CL> { using type = TableCL; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <int K, class TB>

@@ -86,6 +86,7 @@ struct Params {
     const uint32_t *table_g;       // full u32 table (HS variant's cold rows)
     uint32_t hot_rows;             // HS variant: rows cached in shared memory
     const uint32_t *inv;           // internal -> user state ids (renumbered handles), or null
+    uint32_t ncls, cl_magic;       // CL variant: byte classes and ceil(2^32 / ncls)
     uint32_t *user_out;            // optional: the last tile also writes {user state, 0, count lo, hi} here
 };
 

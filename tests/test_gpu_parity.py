@@ -35,17 +35,41 @@ def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
     return res, st
 
 
-VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4, "HS": 5}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4, "HS": 5, "CL": 6}
 
 
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
     return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "H8": n <= 8 and not dfa.bit_mode,
-            "B": n <= 256, "G": True, "HS": not dfa.bit_mode and n <= 32768}[var]
+            "B": n <= 256, "G": True, "HS": not dfa.bit_mode and n <= 32768,
+            "CL": _n_classes(dfa) >= 2 and n * ((_n_classes(dfa) + 1) & ~1) <= 1024}[var]
+
+
+def _n_classes(dfa):
+    """Distinct byte columns of the byte-level (widened in bit mode) table, as the library counts them."""
+    t = dfa.table
+    if dfa.bit_mode:
+        n = t.shape[0]
+        nx = np.zeros((n, 256), np.int64)
+        cnt = np.zeros((n, 256), np.int64)
+        for s in range(n):
+            for c in range(256):
+                q, k = s, 0
+                for i in range(7, -1, -1):
+                    q = int(t[q, (c >> i) & 1])
+                    k += int(dfa.accept[q])
+                nx[s, c], cnt[s, c] = q, k
+        cols = {tuple(nx[:, c]) + tuple(cnt[:, c]) for c in range(256)}
+    else:
+        full = np.full((t.shape[0] + (1 if t.shape[1] < 256 else 0), 256), t.shape[0], np.int64)
+        full[:t.shape[0], :t.shape[1]] = t
+        acc = np.concatenate([dfa.accept, [0] * (full.shape[0] - t.shape[0])]).astype(np.int64)
+        cols = {tuple(full[:, c]) + tuple(acc[full[:, c]]) for c in range(256)}
+    return len(cols)
 
 
 # --------------------------------------------------------------------- worked example on GPU
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS", "CL"])
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
 def test_fig1_worked_example(var, k):
     d = dfas.c_comment(True)
@@ -55,7 +79,7 @@ def test_fig1_worked_example(var, k):
 
 
 # --------------------------------------------------------------------- C1-shaped text
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS", "CL"])
 @pytest.mark.parametrize("chunk", [0, 64, 96, 4096])
 def test_c_comment_text(var, chunk):
     d = dfas.c_comment(True)
@@ -308,3 +332,14 @@ def test_lookback_seqmerge_and_shards(lookback):
             e, c = hit[0] if hit else f.shard_fixup(sh, x)
             x, total = e, total + c
         assert (x, total) == exp
+
+
+@pytest.mark.parametrize("lookback", [0, 64])
+def test_html_all_variants(lookback):
+    d = dfas.html_tokenizer()
+    data = streams.html_bytes(2_500_000, 21)
+    exp = seq.run(d, data)
+    for var in ("CL", "B", "G", "HS"):
+        for k in (1, 2, 4):
+            got, st = gpu_run(d, data, k=k, variant=VARIANTS[var], lookback_len=lookback)
+            assert got == exp, (var, k, lookback, st)

@@ -213,6 +213,8 @@ def main():
     ap.add_argument("--lookback", type=int, default=-1,
                     help="look-back window bytes (R7; -1 = the config's default: c5 0, c1/c4 64, c2/c3 32)")
     ap.add_argument("--chunk", type=int, default=0)
+    ap.add_argument("--eager", type=int, default=0,
+                    help="eager-completion window bytes (NEXT-3): 0 = library default (128), 1 = off, 32..128")
     ap.add_argument("--no-ablation", action="store_true",
                     help="skip the sequential-merge ablation run (Fig. 4a, SURVEY 8.a11)")
     args = ap.parse_args()
@@ -258,7 +260,7 @@ def main():
     f = FSM.from_dfa(d)
     f.set_stream(stream.cuda_stream)
     lookback = w["lookback"]
-    f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback)
+    f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback, eager_window=args.eager)
     res = torch.zeros(4, dtype=torch.int32, device=dev)
     small = total < 4 * 126_000_000
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if small else None
@@ -364,7 +366,7 @@ def main():
     if not args.no_ablation and world == 1:
         # internal ablation: the paper's sequential merge (Fig. 4a) on the same input and chains
         f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_SEQUENTIAL,
-                      lookback_len=lookback)
+                      lookback_len=lookback, eager_window=args.eager)
         f.run_spec_k_async(buf.data_ptr(), nsym, k, res.data_ptr())
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -376,7 +378,7 @@ def main():
         r2 = res.cpu().numpy().view(np.uint32)
         same = (int(r2[0]), int(r2[2]) | (int(r2[3]) << 32)) == final
         f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_PARALLEL,
-                      lookback_len=lookback)
+                      lookback_len=lookback, eager_window=args.eager)
         line["ablation"] = {"sequential_merge_gbs": round(n / ts / 1e9, 3),
                             "parallel_over_sequential": round(ts / step_s, 2), "same_result": same,
                             "paper_v100_context": "2.02-6.74x (P:11, P:53)"}

@@ -133,7 +133,15 @@ typedef struct {
     uint32_t lookback_len;      /* look-back: 0 or 1 = the byte before the chunk; 32..1024 (multiple
                                    of 32) = run the image of the byte before a window of that many bytes
                                    through the window and rank the reached states by multiplicity */
+    uint32_t eager_window;      /* NEXT-3 eager completion: per chunk, the next look-back
+                                   candidates beyond the k speculated ones run in lockstep with the chains
+                                   over the chunk's first eager_window bytes, recording where they meet a
+                                   chain.  0 = default (128), FSM_EAGER_OFF = off, else 32..128 in steps
+                                   of 32.  Results are identical either way; only the re-execution work
+                                   changes. */
 } fsm_options;
+
+#define FSM_EAGER_OFF 1u
 
 int fsm_set_options(fsm_t *f, const fsm_options *opt);
 int fsm_get_options(const fsm_t *f, fsm_options *opt);

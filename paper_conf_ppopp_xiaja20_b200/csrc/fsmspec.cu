@@ -396,12 +396,14 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
+    if (o->eager_window > FSM_EAGER_OFF && (o->eager_window % 32 || o->eager_window > kExtWindow)) return FSM_EINVAL;
     f->opt.chunk_bytes = o->chunk_bytes;            // 0 = adaptive
     f->opt.threads_per_tile = o->threads_per_tile;  // 0 = auto
     f->opt.variant = o->variant;
     f->opt.merge = o->merge;
     f->opt.ctas_per_sm = o->ctas_per_sm;
     f->opt.lookback_len = o->lookback_len;
+    f->opt.eager_window = o->eager_window;
     return FSM_OK;
 }
 
@@ -503,6 +505,7 @@ static int launch_run(fsm *f, const RunSpec &r)
     p.ntiles = ntiles;
     p.k = r.k;
     p.lookback = f->opt.lookback_len > 1 ? f->opt.lookback_len : 0;
+    p.eager_window = f->opt.eager_window == 0 ? kExtWindow : f->opt.eager_window == FSM_EAGER_OFF ? 0u : f->opt.eager_window;
     p.aligned = ((uintptr_t)r.in & 31) == 0;
     p.table = f->d_img[var];
     p.n_states = f->dfa.n;
@@ -557,9 +560,10 @@ static int launch_run(fsm *f, const RunSpec &r)
         const size_t smem_s = std::max<size_t>(16, scratch_offset(var, p.table_bytes));
         CK(cudaFuncSetAttribute((const void *)sf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_s));
         int occ_s = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, sf, kThreads, smem_s));
-        const uint64_t blocks = std::min<uint64_t>((nch + kThreads - 1) / kThreads, (uint64_t)std::max(occ_s, 1) * f->num_sms);
-        sf<<<(uint32_t)blocks, kThreads, smem_s, f->stream>>>(p, f->d_spec);
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, sf, kSpecThreads, smem_s));
+        const uint64_t blocks = std::min<uint64_t>((nch + kSpecThreads - 1) / kSpecThreads,
+                                                   (uint64_t)std::max(occ_s, 1) * f->num_sms);
+        sf<<<(uint32_t)blocks, kSpecThreads, smem_s, f->stream>>>(p, f->d_spec);
         CK(cudaGetLastError());
         p.spec = f->d_spec;
     }
@@ -601,8 +605,7 @@ static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T)
     const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
     if (nch * K > f->seq_cap) {
         cudaStreamSynchronize(f->stream);
-        cudaFree(f->d_spec);
-    cudaFree(f->seq.S);
+        cudaFree(f->seq.S);
         cudaFree(f->seq.E);
         cudaFree(f->seq.C);
         f->seq = SeqBuf{};

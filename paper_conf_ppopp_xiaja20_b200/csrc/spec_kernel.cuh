@@ -13,8 +13,10 @@
 
 namespace speck {
 
+constexpr int kSpecThreads = 1024;  // one CTA per SM when the table image fills shared memory
+
 template <int VAR>
-__global__ void __launch_bounds__(kThreads) spec_kernel(Params p, uint16_t *__restrict__ spec)
+__global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *__restrict__ spec)
 {
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];
@@ -44,8 +46,13 @@ __global__ void __launch_bounds__(kThreads) spec_kernel(Params p, uint16_t *__re
                     const uint32_t byte = (x.w[t >> 2] >> (8 * (t & 3))) & 0xFFu;
                     const typename TB::Row r = tb.row(byte);
                     uint32_t dummy = 0;
+                    // only the image's ni chains are live: skip whole groups of 4 beyond it
 #pragma unroll
-                    for (int i = 0; i < KMAX; i++) y[i] = tb.apply(r, y[i], dummy);
+                    for (int q0 = 0; q0 < KMAX; q0 += 4)
+                        if ((uint32_t)q0 < ni) {
+#pragma unroll
+                            for (int i = q0; i < q0 + 4; i++) y[i] = tb.apply(r, y[i], dummy);
+                        }
                 }
             }
             uint32_t mult[KMAX];

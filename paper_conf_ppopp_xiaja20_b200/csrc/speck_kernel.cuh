@@ -981,7 +981,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
             uint32_t ent[kExt];
 #pragma unroll
             for (int q = 0; q < kExt; q++) ent[q] = kExtNone;
-            if (p.aligned && !empty && e - b >= 32 && Xc[0] != NOSTATE) {
+            if (p.eager_window && p.aligned && !empty && e - b >= 32 && Xc[0] != NOSTATE) {
                 const uint32_t *st32 = reinterpret_cast<const uint32_t *>(smem + L.stash) + j * 8;
                 uint32_t y[K], cy[K], u[kExt], cu[kExt];
                 bool live[kExt];
@@ -999,7 +999,7 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
                     nlive += live[q];
                 }
                 // window: the stashed first 32 bytes, then up to kExtWindow bytes from global (L2)
-                const uint32_t wlen = (uint32_t)((e - b) < kExtWindow ? (e - b) : kExtWindow) & ~31u;
+                const uint32_t wlen = (uint32_t)((e - b) < p.eager_window ? (e - b) : p.eager_window) & ~31u;
 #pragma unroll 1
                 for (uint32_t blk = 0; blk < wlen && nlive > 0; blk += 32) {
                     Bytes32 xb;

@@ -88,6 +88,7 @@ struct Params {
     const uint32_t *inv;           // internal -> user state ids (renumbered handles), or null
     uint32_t ncls, cl_magic;       // CL variant: byte classes and ceil(2^32 / ncls)
     uint32_t *user_out;            // optional: the last tile also writes {user state, 0, count lo, hi} here
+    uint32_t eager_window;         // NEXT-3 eager completion: bytes of lockstep per chunk (0 = off)
 };
 
 }  // namespace speck

@@ -21,6 +21,7 @@ FSM_VARIANT_AUTO, FSM_VARIANT_P4, FSM_VARIANT_P8, FSM_VARIANT_B, FSM_VARIANT_G, 
 FSM_VARIANT_HS, FSM_VARIANT_CL = 5, 6
 VARIANT_NAMES = {0: "P4", 1: "P8", 2: "B", 3: "G", 4: "H8", 5: "HS", 6: "CL"}
 FSM_MERGE_PARALLEL, FSM_MERGE_SEQUENTIAL = 0, 1
+FSM_EAGER_OFF = 1
 
 # every symbol declared in include/fsmspec.h
 EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_set_stream",
@@ -32,7 +33,7 @@ EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_se
 class fsm_options(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
                 ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32),
-                ("lookback_len", ctypes.c_uint32)]
+                ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32)]
 
 
 class fsm_stats(ctypes.Structure):
@@ -176,8 +177,9 @@ class FSM:
         _check(lib().fsm_set_stream(self._h, s), "fsm_set_stream")
 
     def set_options(self, chunk_bytes: int = 0, threads_per_tile: int = 0, variant: int = FSM_VARIANT_AUTO,
-                    merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0, lookback_len: int = 0) -> None:
-        o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm, lookback_len)
+                    merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0, lookback_len: int = 0,
+                    eager_window: int = 0) -> None:
+        o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm, lookback_len, eager_window)
         _check(lib().fsm_set_options(self._h, ctypes.byref(o)), "fsm_set_options")
 
     def options(self) -> dict:

@@ -343,3 +343,35 @@ def test_html_all_variants(lookback):
         for k in (1, 2, 4):
             got, st = gpu_run(d, data, k=k, variant=VARIANTS[var], lookback_len=lookback)
             assert got == exp, (var, k, lookback, st)
+
+
+def test_merge_switch_reuses_window_buffers():
+    """One handle alternating parallel / sequential merge with the window pre-pass, growing the
+    input between calls (the bench's ablation pattern): every result equals the oracle's.  A
+    sequential-merge (re)allocation once freed the pre-pass buffer still in use (illegal access)."""
+    d = dfas.html_tokenizer()
+    data = streams.html_bytes(6_000_000, 33)
+    buf, base = dev(data)
+    with FSM.from_dfa(d) as f:
+        for n in (1_000_000, 3_000_000, 6_000_000):
+            exp = seq.run(d, data[:n])
+            for merge in (fsmspec.FSM_MERGE_PARALLEL, fsmspec.FSM_MERGE_SEQUENTIAL, fsmspec.FSM_MERGE_PARALLEL):
+                f.set_options(lookback_len=64, merge=merge, chunk_bytes=512)
+                assert f.run_spec_k(base, n, 2) == exp, (n, merge)
+        torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("eager", [fsmspec.FSM_EAGER_OFF, 32, 128])
+def test_eager_window_settings(eager):
+    """Eager completion (NEXT-3) off, short and full: identical results, and switching it off
+    cannot reduce the re-execution count (it only ever replaces re-executions)."""
+    cases = [("html", dfas.html_tokenizer(), streams.html_bytes(3_000_000, 41), 2),
+             ("rand64m4", dfas.random_dfa(64, 4, seed=7), streams.splitmix_bytes(9, 0, 2_000_000), 2)]
+    for name, d, data, k in cases:
+        exp = seq.run(d, data)
+        for lb in (0, 64):
+            got, st = gpu_run(d, data, k=k, lookback_len=lb, eager_window=eager, chunk_bytes=1024)
+            assert got == exp, (name, eager, lb, st)
+            if eager == fsmspec.FSM_EAGER_OFF:
+                _, st_on = gpu_run(d, data, k=k, lookback_len=lb, chunk_bytes=1024)
+                assert st["reexec_chunks"] >= st_on["reexec_chunks"], (name, lb, st, st_on)

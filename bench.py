@@ -17,6 +17,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import re
 import statistics
 import subprocess
 import sys
@@ -189,6 +190,7 @@ def run_reference(args, w):
 
 def config_json(args, w):
     return {"workload": w["name"], "input_bytes": w["total"], "k": w["k"], "lookback_len": w.get("lookback"),
+            "eager_window": w.get("eager", 0),
             "n_states": int(w["dfa"].n_states), "parallelism": f"shard{args.gpus}",
             "l2": "input >> L2 (126 MB), no flush needed" if w["total"] > 4 * 126e6 else "L2 flushed between steps"}
 
@@ -215,6 +217,9 @@ def main():
     ap.add_argument("--chunk", type=int, default=0)
     ap.add_argument("--eager", type=int, default=0,
                     help="eager-completion window bytes (NEXT-3): 0 = library default (128), 1 = off, 32..128")
+    ap.add_argument("--tune", action="store_true",
+                    help="NEXT-2: fsm_autotune the look-back and eager windows on a prefix sample before timing")
+    ap.add_argument("--tune-k", action="store_true", help="with --tune: also choose k in [1, min(16, N)]")
     ap.add_argument("--no-ablation", action="store_true",
                     help="skip the sequential-merge ablation run (Fig. 4a, SURVEY 8.a11)")
     args = ap.parse_args()
@@ -260,7 +265,16 @@ def main():
     f = FSM.from_dfa(d)
     f.set_stream(stream.cuda_stream)
     lookback = w["lookback"]
-    f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback, eager_window=args.eager)
+    eager = args.eager
+    w["eager"] = eager
+    f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback, eager_window=eager)
+    tuning = None
+    if args.tune:
+        # offline, like fsm_create (not timed): the measured cost model picks the windows (and k)
+        tuning = f.autotune(buf.data_ptr(), nsym, k_min=0 if args.tune_k else k, k_max=0 if args.tune_k else k)
+        k, lookback, eager = tuning["k"], tuning["lookback_len"], tuning["eager_window"]
+        w["k"], w["lookback"], w["eager"] = k, lookback, eager
+        w["name"] = re.sub(r"spec-\d+", f"spec-{k} (tuned)", w["name"])
     res = torch.zeros(4, dtype=torch.int32, device=dev)
     small = total < 4 * 126_000_000
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if small else None
@@ -363,10 +377,12 @@ def main():
         "stats": {kk: v for kk, v in st.items()},
         "e2e": e2e,
     }
+    if tuning is not None:
+        line["tuning"] = {kk: (round(v, 3) if isinstance(v, float) else v) for kk, v in tuning.items()}
     if not args.no_ablation and world == 1:
         # internal ablation: the paper's sequential merge (Fig. 4a) on the same input and chains
         f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_SEQUENTIAL,
-                      lookback_len=lookback, eager_window=args.eager)
+                      lookback_len=lookback, eager_window=eager)
         f.run_spec_k_async(buf.data_ptr(), nsym, k, res.data_ptr())
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -378,7 +394,7 @@ def main():
         r2 = res.cpu().numpy().view(np.uint32)
         same = (int(r2[0]), int(r2[2]) | (int(r2[3]) << 32)) == final
         f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_PARALLEL,
-                      lookback_len=lookback, eager_window=args.eager)
+                      lookback_len=lookback, eager_window=eager)
         line["ablation"] = {"sequential_merge_gbs": round(n / ts / 1e9, 3),
                             "parallel_over_sequential": round(ts / step_s, 2), "same_result": same,
                             "paper_v100_context": "2.02-6.74x (P:11, P:53)"}

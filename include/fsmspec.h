@@ -197,6 +197,58 @@ void fsm_shard_free(fsm_shard_t *state);  /* NULL is a no-op */
  * (delayed strategy).  out may alias a or b. */
 int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, fsm_shard_map *out);
 
+/* ------------------------------------------------------------- NEXT-2: k / look-back tuning ---
+ * The paper leaves the choice of k to the user and names a cost model for it as future work
+ * (Figs. 12-13, show the best k differs by FSM and input).  fsm_autotune picks
+ * k, the look-back window (reading R7) and the eager-completion window (NEXT-3) for one
+ * DFA and input by timing the real kernel on a prefix sample of the input -- a measured cost
+ * model: every candidate's cost is its own sampled time, which already includes its sampled
+ * re-execution (miss) rate.  The search is staged: (1) every instantiated k in [k_min, k_max] with the
+ * default window (64 bytes, eager on) and with the paper's depth-1 look-back (eager off); (2) for
+ * the two fastest k, look-back windows {0, 32, 64, 128, 256} x eager {off, 128}.
+ *   input, len   device pointer and length (symbols) of the input the runs will process
+ *   k_min, k_max smallest / largest k to consider (0 = 1 / min(FSM_KMAX, n_states); k_min = k_max
+ *                tunes only the windows for that k)
+ *   sample_len   symbols timed per candidate (0 = min(len, 2 GiB)); the prefix is used, run with the
+ *                chunk and tile geometry of the full length so its cost per byte is the full run's
+ *   out          the choice and its evidence; the chosen lookback_len / eager_window are also
+ *                written into the handle's options (the caller passes out->k to the runs)
+ * Results of runs are identical under every setting; only speed changes.  Synchronises the
+ * handle's stream.  Errors: FSM_EINVAL, FSM_ECUDA. */
+typedef struct {
+    uint32_t k;                 /* chosen k */
+    uint32_t lookback_len;      /* chosen look-back window (0 = depth-1 look-back) */
+    uint32_t eager_window;      /* chosen eager-completion window (FSM_EAGER_OFF = off) */
+    uint32_t candidates;        /* configurations timed */
+    uint64_t sample_len;        /* symbols per timed run */
+    double best_gbs;            /* sample bytes / median time of the chosen configuration */
+    double paper_gbs;           /* same for the paper's plain setting: k = 1, depth-1 look-back, no eager */
+    double hit_rate;            /* 1 - re-executed chunks / chunks, chosen configuration */
+} fsm_tuning;
+
+int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k_min, uint32_t k_max,
+                 uint64_t sample_len, fsm_tuning *out);
+
+/* -------------------------------------------------- NEXT-4: many FSMs over one resident input ---
+ * The network-intrusion case the paper uses to justify amortised layout work: M
+ * DFAs scan the same input.  fsm_run_multi computes, for each DFA i, exactly what
+ * fsm_run_spec_k(fsms[i], input, len, k[i]) computes, in fused launches: DFAs with the same table
+ * variant and instantiated K share one persistent grid, whose CTAs take (tile, DFA) pairs in
+ * tile-major order so that the input is read from HBM about once per group (the other DFAs hit
+ * the tile in L2).  Each handle's own options (look-back, eager window) apply; the chunk and tile
+ * geometry are the first handle of each group's.
+ *   fsms, m        1 <= m <= FSM_MULTI_MAX distinct handles, same input mode and device; the work is
+ *                  enqueued on fsms[0]'s stream
+ *   input, len     as fsm_run_spec_k (one input for all)
+ *   k              m values, each valid for its handle
+ *   final_states, accept_counts   m results each (user state ids)
+ * Blocks until the results are on the host; each handle's fsm_get_stats describes its own run.
+ * Errors: FSM_EINVAL, FSM_ECUDA; FSM_ESYMBOL if any DFA saw an out-of-alphabet byte (results are
+ * still written; that DFA's final state is then n_states). */
+#define FSM_MULTI_MAX 64u
+int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *input, uint64_t len, const uint32_t *k,
+                  uint32_t *final_states, uint64_t *accept_counts);
+
 /* ----------------------------------------------------------------------- host-only helpers ---
  * fsm_lookback_table: the look-back speculation table the library builds at fsm_create (host
  * code, no GPU needed).  For every input byte c: the image {delta(s, c)} (bit mode: of the

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -33,11 +34,13 @@ typedef void (*FixFn)(FixParams);
 typedef void (*SeqLocalFn)(Params, SeqBuf);
 typedef void (*SeqWalkFn)(Params, SeqBuf);
 typedef void (*SpecFn)(Params, uint16_t *);
+typedef void (*MultiFn)(Params, const Params *, uint32_t);
 
 // Kernel instantiations live in one translation unit per table variant (kernels_*.cu, compiled in
 // parallel); each exports these accessors.
 #define FSM_DECLARE_VARIANT(NAME)                                   \
     KernelFn get_kernel_##NAME(int K);                              \
+    MultiFn get_multi_##NAME(int K);                                \
     FixFn get_fix_##NAME();                                         \
     void get_seq_##NAME(int K, SeqLocalFn &l, SeqWalkFn &w);       \
     SpecFn get_spec_##NAME();
@@ -59,6 +62,18 @@ static KernelFn get_kernel(int var, int K)
     case VAR_CL: return get_kernel_cl(K);
     case VAR_B: return get_kernel_b(K);
     default: return get_kernel_g(K);
+    }
+}
+static MultiFn get_multi(int var, int K)
+{
+    switch (var) {
+    case VAR_P4: return get_multi_p4(K);
+    case VAR_P8: return get_multi_p8(K);
+    case VAR_H8: return get_multi_h8(K);
+    case VAR_HS: return get_multi_hs(K);
+    case VAR_CL: return get_multi_cl(K);
+    case VAR_B: return get_multi_b(K);
+    default: return get_multi_g(K);
     }
 }
 static FixFn get_fix(int var)
@@ -146,6 +161,9 @@ struct fsm {
     // look-back window pre-pass output
     uint16_t *d_spec = nullptr;
     size_t spec_cap = 0;
+    // multi-FSM groups led by this handle: per-DFA Params in device memory
+    Params *d_multi = nullptr;
+    size_t multi_cap = 0;
     // sequential-merge ablation buffers
     SeqBuf seq{};
     size_t seq_cap = 0;
@@ -220,6 +238,7 @@ static void free_all(fsm *f)
     cudaFree(f->d_stage[0]);
     cudaFree(f->d_stage[1]);
     cudaFree(f->d_spec);
+    cudaFree(f->d_multi);
     cudaFree(f->seq.S);
     cudaFree(f->seq.E);
     cudaFree(f->seq.C);
@@ -434,6 +453,8 @@ struct RunSpec {
     DevResult *result;
     int force_variant;     // -1 = handle options
     uint32_t merge;
+    uint64_t geom_len_bytes = 0;  // geometry as for a run of this many bytes (0 = len): tuning samples
+    uint32_t force_T = 0, force_chunk = 0;  // multi-FSM groups: one geometry for every DFA
 };
 
 static int variant_of(const fsm *f, int force, uint32_t k = 1)
@@ -482,14 +503,25 @@ static int ensure_desc(fsm *f, size_t ntiles)
 
 static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T);
 
-static int launch_run(fsm *f, const RunSpec &r)
+// Everything of a run but the fused kernel's launch: variant, geometry, Params, the look-back
+// pre-pass (launched here), descriptors.  Shared by single runs and multi-FSM groups.
+struct Prepared {
+    Params p;
+    int var, K;
+    uint32_t T;
+    size_t smem;
+};
+
+static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
 {
     const int var = variant_of(f, r.force_variant, r.k);
     const int K = kslots(r.k);
     const bool bits = f->mode == FSM_INPUT_BITS_MSB;
     const uint64_t len_bytes = bits ? r.len_sym / 8 : r.len_sym;
     uint32_t T = 0, chunk = 0;
-    pick_geometry(f, len_bytes, K, T, chunk);
+    pick_geometry(f, r.geom_len_bytes ? std::max(r.geom_len_bytes, len_bytes) : len_bytes, K, T, chunk);
+    if (r.force_T) T = r.force_T;
+    if (r.force_chunk) chunk = r.force_chunk;
     if (r.merge == FSM_MERGE_SEQUENTIAL) T = std::min<uint32_t>(T, kThreads);
     const uint64_t tile_bytes = (uint64_t)T * chunk;
     uint64_t ntiles64 = (len_bytes + tile_bytes - 1) / tile_bytes;
@@ -568,27 +600,17 @@ static int launch_run(fsm *f, const RunSpec &r)
         p.spec = f->d_spec;
     }
 
-    if (r.merge == FSM_MERGE_SEQUENTIAL) {
-        if (r.keyed) return FSM_EINVAL;
-        return launch_seq(f, p, var, K, T);
-    }
-
+    out.p = p;
+    out.var = var;
+    out.K = K;
+    out.T = T;
+    out.smem = smem;
+    if (r.merge == FSM_MERGE_SEQUENTIAL) return FSM_OK;
     if ((rc = ensure_desc(f, ntiles))) return rc;
-    p.desc = f->d_desc;
-    KernelFn fn = get_kernel(var, K);
-    CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    int occ = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)T, smem));
-    if (occ < 1) return FSM_EINVAL;
-    if (f->opt.ctas_per_sm) occ = std::min<int>(occ, (int)f->opt.ctas_per_sm);
-    const uint32_t grid = (uint32_t)std::min<uint64_t>(ntiles, (uint64_t)occ * f->num_sms);
+    out.p.desc = f->d_desc;
     f->epoch = (f->epoch + 1) & 0x3FFFFFFFu;
     if (f->epoch == 0) f->epoch = 1;
-    p.epoch = f->epoch;
-    p.ticket_base = f->ticket_base;
-    fn<<<grid, T, smem, f->stream>>>(p);
-    CK(cudaGetLastError());
-    f->ticket_base += ntiles + grid;  // every CTA takes one ticket past the end
+    out.p.epoch = f->epoch;
     f->last.chunks = (len_bytes + chunk - 1) / chunk;
     f->last.tiles = ntiles;
     f->last.chunk_bytes = chunk;
@@ -596,6 +618,35 @@ static int launch_run(fsm *f, const RunSpec &r)
     f->last.variant = var;
     f->last.k_slots = K;
     f->last.lookback_len = p.lookback;
+    return FSM_OK;
+}
+
+static int launch_run(fsm *f, const RunSpec &r)
+{
+    Prepared pr;
+    int rc = prepare_run(f, r, pr);
+    if (rc) return rc;
+    Params p = pr.p;
+    const int var = pr.var, K = pr.K;
+    const uint32_t T = pr.T;
+    const size_t smem = pr.smem;
+    if (r.merge == FSM_MERGE_SEQUENTIAL) {
+        if (r.keyed) return FSM_EINVAL;
+        return launch_seq(f, p, var, K, T);
+    }
+
+    KernelFn fn = get_kernel(var, K);
+    CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)T, smem));
+    if (occ < 1) return FSM_EINVAL;
+    if (f->opt.ctas_per_sm) occ = std::min<int>(occ, (int)f->opt.ctas_per_sm);
+    const uint32_t ntiles = p.ntiles;
+    const uint32_t grid = (uint32_t)std::min<uint64_t>(ntiles, (uint64_t)occ * f->num_sms);
+    p.ticket_base = f->ticket_base;
+    fn<<<grid, T, smem, f->stream>>>(p);
+    CK(cudaGetLastError());
+    f->ticket_base += ntiles + grid;  // every CTA takes one ticket past the end
     return FSM_OK;
 }
 
@@ -865,4 +916,228 @@ extern "C" int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, f
     }
     *out = r;
     return FSM_OK;
+}
+
+// ------------------------------------------------------------------ NEXT-2: autotuning -------
+// Staged measured search (include/fsmspec.h): the cost of a candidate is its median sampled time.
+namespace {
+struct TuneCand {
+    uint32_t k, lookback, eager;
+    double ms = 0, hit = 0;
+};
+}  // namespace
+
+static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom_len, TuneCand &c, cudaEvent_t e0,
+                          cudaEvent_t e1)
+{
+    fsm_options o = f->opt;
+    o.lookback_len = c.lookback;
+    o.eager_window = c.eager;
+    o.merge = FSM_MERGE_PARALLEL;
+    int rc = fsm_set_options(f, &o);
+    if (rc) return rc;
+    // warm-up run, synchronous: also yields the sampled success rate
+    RunSpec r{nullptr, in, len, c.k, false, 0, f->start_int, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL, geom_len};
+    if ((rc = launch_run(f, r))) return rc;
+    if ((rc = finish_sync(f, f->d_result))) return rc;
+    c.hit = f->last.chunks ? 1.0 - (double)f->last.reexec_chunks / (double)f->last.chunks : 1.0;
+    float t[3];
+    for (int i = 0; i < 3; i++) {
+        CK(cudaEventRecord(e0, f->stream));
+        if ((rc = launch_run(f, r))) return rc;
+        CK(cudaEventRecord(e1, f->stream));
+        CK(cudaEventSynchronize(e1));
+        CK(cudaEventElapsedTime(&t[i], e0, e1));
+    }
+    std::sort(t, t + 3);
+    c.ms = t[1];
+    return FSM_OK;
+}
+
+extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k_min, uint32_t k_max,
+                            uint64_t sample_len, fsm_tuning *out)
+{
+    if (!f || !out || (len > 0 && !input)) return FSM_EINVAL;
+    const uint32_t kcap = std::min<uint32_t>(FSM_KMAX, f->n_user);
+    if (k_max == 0 || k_max > kcap) k_max = kcap;
+    if (k_min == 0) k_min = 1;
+    if (k_min > k_max) return FSM_EINVAL;
+    const bool bits = f->mode == FSM_INPUT_BITS_MSB;
+    const uint64_t sym_per_byte = bits ? 8 : 1;
+    // default sample: 2 GiB -- several waves of full-size tiles over every SM, run with the
+    // geometry (chunk, tile) of the full input so that the sampled cost is the full run's per byte
+    if (sample_len == 0) sample_len = ((uint64_t)2 << 30) * sym_per_byte;
+    const uint64_t n = std::min(len, sample_len);
+    const fsm_options saved = f->opt;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    CK(cudaEventCreate(&e0));
+    CK(cudaEventCreate(&e1));
+    std::vector<TuneCand> tried;
+    int rc = FSM_OK;
+    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg) -> int {
+        for (const TuneCand &c : tried)
+            if (c.k == k && c.lookback == lb && c.eager == eg) return FSM_OK;
+        TuneCand c{k, lb, eg};
+        int r = time_candidate(f, input, n, len / sym_per_byte, c, e0, e1);
+        if (r == FSM_OK) tried.push_back(c);
+        return r;
+    };
+    // stage 1: every instantiated k with the default window and with the paper's setting
+    std::vector<uint32_t> ks;
+    for (int i = 0; i < kNumKs; i++)
+        if ((uint32_t)kKs[i] >= k_min && (uint32_t)kKs[i] <= k_max) ks.push_back((uint32_t)kKs[i]);
+    if (ks.empty() || ks[0] != k_min) ks.insert(ks.begin(), k_min);
+    if (ks.back() != k_max) ks.push_back(k_max);
+    for (uint32_t k : ks) {
+        if ((rc = run(k, 64, 0))) break;
+        if ((rc = run(k, 0, FSM_EAGER_OFF))) break;
+    }
+    // stage 2: windows x eager for the two fastest k
+    if (rc == FSM_OK) {
+        std::vector<TuneCand> s1 = tried;
+        std::sort(s1.begin(), s1.end(), [](const TuneCand &a, const TuneCand &b) { return a.ms < b.ms; });
+        std::vector<uint32_t> best_k;
+        for (const TuneCand &c : s1)
+            if (best_k.size() < 2 && std::find(best_k.begin(), best_k.end(), c.k) == best_k.end()) best_k.push_back(c.k);
+        static const uint32_t lbs[] = {0, 32, 64, 128, 256};
+        for (uint32_t k : best_k)
+            for (uint32_t lb : lbs)
+                for (uint32_t eg : {FSM_EAGER_OFF, 0u})
+                    if (rc == FSM_OK) rc = run(k, lb, eg);
+    }
+    if (rc == FSM_OK) rc = run(1, 0, FSM_EAGER_OFF);  // the paper's plain spec-1, for reference
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    f->opt = saved;
+    if (rc) return rc;
+    const TuneCand *best = nullptr;  // the paper's reference point may lie outside [k_min, k_max]
+    for (const TuneCand &c : tried)
+        if (c.k >= k_min && c.k <= k_max && (!best || c.ms < best->ms)) best = &c;
+    const double bytes = (double)n / (double)sym_per_byte;
+    double paper_ms = 0;
+    for (const TuneCand &c : tried)
+        if (c.k == 1 && c.lookback == 0 && c.eager == FSM_EAGER_OFF) paper_ms = c.ms;
+    out->k = best->k;
+    out->lookback_len = best->lookback;
+    out->eager_window = best->eager == 0 ? kExtWindow : best->eager;
+    out->candidates = (uint32_t)tried.size();
+    out->sample_len = n;
+    out->best_gbs = best->ms > 0 ? bytes / (best->ms * 1e6) : 0.0;
+    out->paper_gbs = paper_ms > 0 ? bytes / (paper_ms * 1e6) : 0.0;
+    out->hit_rate = best->hit;
+    f->opt.lookback_len = best->lookback;
+    f->opt.eager_window = out->eager_window;
+    return FSM_OK;
+}
+
+// --------------------------------------------------------- NEXT-4: many FSMs, one input ------
+// DFAs are grouped by (table variant, K); each group is one fused launch (speck_multi_kernel) led
+// by fsms[0]: its stream, ticket counter and Params buffer.  Every handle keeps its own
+// descriptors, result and counters.
+extern "C" int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *input, uint64_t len, const uint32_t *k,
+                             uint32_t *final_states, uint64_t *accept_counts)
+{
+    if (!fsms || m == 0 || m > FSM_MULTI_MAX || !k || !final_states || !accept_counts) return FSM_EINVAL;
+    fsm *lead = fsms[0];
+    for (uint32_t i = 0; i < m; i++) {
+        int rc = check_run_args(fsms[i], input, len, k[i]);
+        if (rc) return rc;
+        if (fsms[i]->mode != lead->mode || fsms[i]->device != lead->device) return FSM_EINVAL;
+        for (uint32_t j = 0; j < i; j++)
+            if (fsms[j] == fsms[i]) return FSM_EINVAL;  // one result slot per handle
+    }
+    const bool bits = lead->mode == FSM_INPUT_BITS_MSB;
+    const uint64_t len_bytes = bits ? len / 8 : len;
+    // every handle runs on the leader's stream for this call
+    std::vector<cudaStream_t> saved(m);
+    for (uint32_t i = 0; i < m; i++) {
+        saved[i] = fsms[i]->stream;
+        fsms[i]->stream = lead->stream;
+    }
+    auto restore = [&]() {
+        for (uint32_t i = 0; i < m; i++) fsms[i]->stream = saved[i];
+    };
+    if (lead->multi_cap < m) {
+        cudaStreamSynchronize(lead->stream);
+        cudaFree(lead->d_multi);
+        lead->d_multi = nullptr;
+        lead->multi_cap = 0;
+        if (cudaMalloc(&lead->d_multi, m * sizeof(Params)) != cudaSuccess) {
+            restore();
+            return FSM_ECUDA;
+        }
+        lead->multi_cap = m;
+    }
+    std::vector<int> group_of(m, -1);
+    std::vector<Params> hp(m);
+    int rc = FSM_OK;
+    uint32_t base = 0;
+    for (uint32_t i = 0; i < m && rc == FSM_OK; i++) {
+        if (group_of[i] >= 0) continue;
+        const int var = variant_of(fsms[i], -1, k[i]);
+        const int K = kslots(k[i]);
+        std::vector<uint32_t> g;
+        for (uint32_t j = i; j < m; j++)
+            if (group_of[j] < 0 && variant_of(fsms[j], -1, k[j]) == var && kslots(k[j]) == K) {
+                group_of[j] = (int)i;
+                g.push_back(j);
+            }
+        uint32_t T = 0, chunk = 0;
+        pick_geometry(fsms[i], len_bytes, K, T, chunk);
+        size_t smem = 0;
+        uint32_t tbytes = 0;
+        for (uint32_t n = 0; n < g.size() && rc == FSM_OK; n++) {
+            fsm *f = fsms[g[n]];
+            RunSpec r{nullptr, input, len, k[g[n]], false, 0, f->start_int, nullptr, f->d_result, var,
+                      FSM_MERGE_PARALLEL, 0, T, chunk};
+            Prepared pr;
+            if ((rc = prepare_run(f, r, pr))) break;
+            hp[base + n] = pr.p;
+            smem = std::max(smem, pr.smem);
+            tbytes = std::max(tbytes, pr.p.table_bytes);
+        }
+        if (rc) break;
+        const uint32_t M = (uint32_t)g.size();
+        Params gp = hp[base];
+        gp.table_bytes = tbytes;
+        if ((uint64_t)gp.ntiles * M > 0x7FFFFFFFull) {
+            rc = FSM_EINVAL;
+            break;
+        }
+        if (cudaMemcpyAsync(lead->d_multi + base, hp.data() + base, M * sizeof(Params), cudaMemcpyHostToDevice,
+                            lead->stream) != cudaSuccess) {
+            rc = FSM_ECUDA;
+            break;
+        }
+        MultiFn fn = get_multi(var, K);
+        int occ = 0;
+        if (cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess ||
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)T, smem) != cudaSuccess || occ < 1) {
+            rc = FSM_ECUDA;
+            break;
+        }
+        if (lead->opt.ctas_per_sm) occ = std::min<int>(occ, (int)lead->opt.ctas_per_sm);
+        const uint64_t ntickets = (uint64_t)gp.ntiles * M;
+        const uint32_t grid = (uint32_t)std::min<uint64_t>(ntickets, (uint64_t)occ * lead->num_sms);
+        gp.ticket = lead->d_ticket;
+        gp.ticket_base = lead->ticket_base;
+        fn<<<grid, T, smem, lead->stream>>>(gp, lead->d_multi + base, M);
+        if (cudaGetLastError() != cudaSuccess) {
+            rc = FSM_ECUDA;
+            break;
+        }
+        lead->ticket_base += (uint32_t)ntickets + grid;
+        base += M;
+    }
+    bool esym = false;
+    for (uint32_t i = 0; i < m && rc == FSM_OK; i++) {
+        fsm *f = fsms[i];
+        if ((rc = finish_sync(f, f->d_result))) break;
+        if (is_sink(f, f->h_result->final_state)) esym = true;
+        final_states[i] = to_user(f, f->h_result->final_state);
+        accept_counts[i] = f->h_result->count;
+    }
+    restore();
+    if (rc) return rc;
+    return esym ? FSM_ESYMBOL : FSM_OK;
 }

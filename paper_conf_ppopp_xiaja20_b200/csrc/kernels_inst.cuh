@@ -12,6 +12,7 @@ typedef void (*FixFn)(FixParams);
 typedef void (*SeqLocalFn)(Params, SeqBuf);
 typedef void (*SeqWalkFn)(Params, SeqBuf);
 typedef void (*SpecFn)(Params, uint16_t *);
+typedef void (*MultiFn)(Params, const Params *, uint32_t);
 
 #define FSM_CAT2(a, b) a##b
 #define FSM_CAT(a, b) FSM_CAT2(a, b)
@@ -27,6 +28,20 @@ KernelFn FSM_CAT(get_kernel_, FSM_VAR_NAME)(int K)
     case 8: return speck_kernel<8, FSM_VAR>;
     case 12: return speck_kernel<12, FSM_VAR>;
     default: return speck_kernel<16, FSM_VAR>;
+    }
+}
+
+MultiFn FSM_CAT(get_multi_, FSM_VAR_NAME)(int K)
+{
+    switch (K) {
+    case 1: return speck_multi_kernel<1, FSM_VAR>;
+    case 2: return speck_multi_kernel<2, FSM_VAR>;
+    case 3: return speck_multi_kernel<3, FSM_VAR>;
+    case 4: return speck_multi_kernel<4, FSM_VAR>;
+    case 6: return speck_multi_kernel<6, FSM_VAR>;
+    case 8: return speck_multi_kernel<8, FSM_VAR>;
+    case 12: return speck_multi_kernel<12, FSM_VAR>;
+    default: return speck_multi_kernel<16, FSM_VAR>;
     }
 }
 

@@ -908,8 +908,15 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
 }
 
 // ------------------------------------------------------------------------------- the kernel --
-template <int K, int VAR>
-__global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Params p)
+// The body serves two kernels.  speck_kernel: one DFA, parameters in the kernel parameter space.
+// speck_multi_kernel (NEXT-4, many FSMs over one resident input): M DFAs of the same
+// table variant and K share one persistent grid and one ticket counter; ticket t is tile t / M of
+// DFA t % M, so the M CTAs that run the same input tile for different DFAs run at about the same
+// time and the tile is read from HBM once and from L2 M - 1 times.  Each DFA keeps its own
+// descriptors (its own decoupled look-back), result and counters (pm[d]); a CTA reloads the table
+// image into shared memory when its ticket switches DFA.
+template <int K, int VAR, bool MULTI>
+__device__ __forceinline__ void speck_body(const Params &p0, const Params *__restrict__ pm, uint32_t M)
 {
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];  // no static shared memory: see kSmemWindowBase
@@ -918,10 +925,11 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = T >> 5;
     const uint32_t j = threadIdx.x;
 
-    const Layout L(T, K, scratch_offset(VAR, p.table_bytes));
+    // MULTI: p0.table_bytes is the group's largest table image, so one layout serves every DFA
+    const Layout L(T, K, scratch_offset(VAR, p0.table_bytes));
     check_smem_window(VAR, L.total);
     TB tb;
-    tb.setup(smem, p.table, p.n_states, kconst(p));
+    if (!MULTI) tb.setup(smem, p0.table, p0.n_states, kconst(p0));
     uint32_t *Qe = reinterpret_cast<uint32_t *>(smem + L.qe);
     uint32_t *Qc = reinterpret_cast<uint32_t *>(smem + L.qc);
     uint16_t *Sj = reinterpret_cast<uint16_t *>(smem + L.sj);
@@ -931,17 +939,26 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
     uint32_t *wI = reinterpret_cast<uint32_t *>(smem + L.wi);
     uint32_t &s_tile = *reinterpret_cast<uint32_t *>(smem + L.misc);
     uint32_t *Ext = reinterpret_cast<uint32_t *>(smem + L.ext);
-
-    const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
-    const unsigned long long start_count = p.start_dev ? p.start_dev->count : 0ull;
-    const uint32_t ksel = p.k;
+    const uint32_t ntickets = MULTI ? p0.ntiles * M : p0.ntiles;
+    uint32_t loaded = 0xFFFFFFFFu;  // MULTI: DFA whose table image is in shared memory
 
     for (;;) {
         __syncthreads();  // smem reuse across tiles; also orders the table setup
-        if (threadIdx.x == 0) s_tile = atomicAdd(p.ticket, 1u) - p.ticket_base;
+        if (threadIdx.x == 0) s_tile = atomicAdd(p0.ticket, 1u) - p0.ticket_base;
         __syncthreads();
-        const uint32_t tile = s_tile;
-        if (tile >= p.ntiles) break;
+        const uint32_t ticket = s_tile;
+        if (ticket >= ntickets) break;
+        const uint32_t dfa = MULTI ? ticket % M : 0u;
+        const uint32_t tile = MULTI ? ticket / M : ticket;
+        const Params &p = MULTI ? pm[dfa] : p0;
+        if (MULTI && dfa != loaded) {  // block-uniform
+            tb.setup(smem, p.table, p.n_states, kconst(p));
+            loaded = dfa;
+            __syncthreads();
+        }
+        const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
+        const unsigned long long start_count = p.start_dev ? p.start_dev->count : 0ull;
+        const uint32_t ksel = p.k;
 
         const uint64_t tile_base = (uint64_t)tile * T * p.chunk;
         const uint64_t b = tile_base + (uint64_t)j * p.chunk;
@@ -1339,6 +1356,19 @@ __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Pa
             }
         }
     }
+}
+
+template <int K, int VAR>
+__global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Params p)
+{
+    speck_body<K, VAR, false>(p, nullptr, 1);
+}
+
+template <int K, int VAR>
+__global__ void __launch_bounds__(max_threads(K), min_blocks(K))
+    speck_multi_kernel(Params g, const Params *__restrict__ pm, uint32_t M)
+{
+    speck_body<K, VAR, true>(g, pm, M);
 }
 
 }  // namespace speck

@@ -27,13 +27,19 @@ FSM_EAGER_OFF = 1
 EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_set_stream",
            "fsm_run_spec_k", "fsm_run_spec_k_async", "fsm_run_spec_k_host", "fsm_set_options",
            "fsm_get_options", "fsm_get_stats", "fsm_run_shard", "fsm_shard_fixup", "fsm_shard_free",
-           "fsm_map_compose", "fsm_lookback_table", "fsm_version")
+           "fsm_map_compose", "fsm_lookback_table", "fsm_version", "fsm_autotune", "fsm_run_multi")
 
 
 class fsm_options(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
                 ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32),
                 ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32)]
+
+
+class fsm_tuning(ctypes.Structure):
+    _fields_ = [("k", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32),
+                ("candidates", ctypes.c_uint32), ("sample_len", ctypes.c_uint64), ("best_gbs", ctypes.c_double),
+                ("paper_gbs", ctypes.c_double), ("hit_rate", ctypes.c_double)]
 
 
 class fsm_stats(ctypes.Structure):
@@ -95,6 +101,9 @@ def lib() -> ctypes.CDLL:
                                        ctypes.POINTER(fsm_shard_map)]),
             "fsm_lookback_table": (_I32, [_P, _U32, _U32, _U32, _P, _P]),
             "fsm_version": (ctypes.c_char_p, []),
+            "fsm_run_multi": (_I32, [ctypes.POINTER(_P), _U32, _P, _U64, ctypes.POINTER(_U32), ctypes.POINTER(_U32),
+                                     ctypes.POINTER(_U64)]),
+            "fsm_autotune": (_I32, [_P, _P, _U64, _U32, _U32, _U64, ctypes.POINTER(fsm_tuning)]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(l, name)
@@ -212,6 +221,14 @@ class FSM:
                "fsm_run_spec_k_host")
         return int(q.value), int(n.value)
 
+    def autotune(self, inp, length: int, k_min: int = 0, k_max: int = 0, sample_len: int = 0) -> dict:
+        """fsm_autotune (NEXT-2): choose k, look-back window and eager window by timing the kernel on
+        a prefix sample; the chosen windows are applied to this handle, the chosen k is returned."""
+        t = fsm_tuning()
+        _check(lib().fsm_autotune(self._h, _ptr(inp), length, k_min, k_max, sample_len, ctypes.byref(t)), "fsm_autotune")
+        return {n: (float(getattr(t, n)) if isinstance(getattr(t, n), float) else int(getattr(t, n)))
+                for n, _ in t._fields_}
+
     def run_shard(self, inp, length: int, halo=None, halo_len: int = 0, k: int = 1, keep: bool = False):
         """fsm_run_shard -> (fsm_shard_map, shard handle or None)."""
         m = fsm_shard_map()
@@ -238,3 +255,15 @@ class Shard:
         self._h = None
 
     __del__ = close
+
+
+def run_multi(fsms, inp, length: int, ks) -> list[tuple[int, int]]:
+    """fsm_run_multi (NEXT-4): every FSM of ``fsms`` over the same device-resident input, fused per
+    (variant, K) group; returns [(final_state, accept_count)] in order."""
+    m = len(fsms)
+    hs = (_P * m)(*[f._h for f in fsms])
+    kk = (_U32 * m)(*ks)
+    q = (_U32 * m)()
+    n = (_U64 * m)()
+    _check(lib().fsm_run_multi(hs, m, _ptr(inp), length, kk, q, n), "fsm_run_multi")
+    return [(int(q[i]), int(n[i])) for i in range(m)]

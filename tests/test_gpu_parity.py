@@ -375,3 +375,56 @@ def test_eager_window_settings(eager):
             if eager == fsmspec.FSM_EAGER_OFF:
                 _, st_on = gpu_run(d, data, k=k, lookback_len=lb, chunk_bytes=1024)
                 assert st["reexec_chunks"] >= st_on["reexec_chunks"], (name, lb, st, st_on)
+
+
+def test_autotune_choice_is_exact_and_not_slower():
+    """NEXT-2: fsm_autotune times candidates on a prefix sample and applies the fastest windows; the
+    run with the chosen k and options equals the oracle, and the choice is never slower (on the
+    sample) than the paper's plain setting it also timed."""
+    cases = [("html", dfas.html_tokenizer(), streams.html_bytes(24_000_000, 51), 0, 0),
+             ("rand16m2", dfas.random_dfa(16, 2, seed=3), streams.splitmix_bytes(4, 0, 16_000_000), 0, 4),
+             ("rand64m4-fixedk", dfas.random_dfa(64, 4, seed=5), streams.splitmix_bytes(6, 0, 8_000_000), 2, 2)]
+    for name, d, data, kmin, kmax in cases:
+        exp = seq.run(d, data)
+        buf, ptr = dev(data)
+        with FSM.from_dfa(d) as f:
+            t = f.autotune(ptr, data.size, k_min=kmin, k_max=kmax, sample_len=8_000_000)
+            assert t["candidates"] >= 3 and 0.0 <= t["hit_rate"] <= 1.0, (name, t)
+            assert t["best_gbs"] >= t["paper_gbs"] > 0 or kmin > 1, (name, t)
+            if kmin:
+                assert t["k"] == kmin
+            o = f.options()
+            assert o["lookback_len"] == t["lookback_len"] and o["eager_window"] == t["eager_window"]
+            assert f.run_spec_k(ptr, data.size, t["k"]) == exp, (name, t)
+        torch.cuda.synchronize()
+
+
+def test_run_multi_matches_single_runs():
+    """NEXT-4: many FSMs over one resident input.  fsm_run_multi fuses DFAs of the same variant and
+    K into one launch; every DFA's result equals the oracle, across mixed variants (P4, P8, B, CL,
+    HS/G), mixed k, per-handle look-back options and a ragged length."""
+    data = streams.html_bytes(5_000_003, 61)
+    buf, ptr = dev(data)
+    dfa_list = [dfas.html_tokenizer(), dfas.random_dfa(8, 2, seed=1), dfas.random_dfa(8, 3, seed=2),
+                dfas.c_comment(True), dfas.random_dfa(16, 2, seed=3), dfas.random_dfa(200, 4, seed=4),
+                dfas.random_dfa(8, 2, seed=5), dfas.aho_corasick(dfas.snort_patterns(300, seed=6))]
+    ks = [1, 2, 2, 1, 2, 4, 2, 1]
+    exp = [seq.run(d, data) for d in dfa_list]
+    fs = [FSM.from_dfa(d) for d in dfa_list]
+    try:
+        fs[0].set_options(lookback_len=64)
+        fs[4].set_options(lookback_len=32, eager_window=fsmspec.FSM_EAGER_OFF)
+        got = fsmspec.run_multi(fs, ptr, data.size, ks)
+        assert got == exp
+        # stats describe each handle's own run
+        for f in fs:
+            assert f.stats()["chunks"] > 0
+        # a second call on the same handles (epochs, tickets advance) and a sub-group
+        assert fsmspec.run_multi(fs[1:3] + fs[6:7], ptr, 4_000_000, [2, 2, 2]) == \
+            [seq.run(d, data[:4_000_000]) for d in (dfa_list[1], dfa_list[2], dfa_list[6])]
+        with pytest.raises(fsmspec.FsmError):
+            fsmspec.run_multi([fs[1], fs[1]], ptr, data.size, [1, 1])
+    finally:
+        for f in fs:
+            f.close()
+        torch.cuda.synchronize()

@@ -8,7 +8,7 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-SO = os.path.join(HERE, "libfsmspec.so")
+SO = os.environ.get("FSMSPEC_BUILD_SO") or os.path.join(HERE, "libfsmspec.so")  # override: experiments only
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
@@ -39,7 +39,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
     def unit(u):
         obj = os.path.join(tmp, u + ".o")
-        cmd = [NVCC, *FLAGS, "-I", os.path.join(ROOT, "include"), "-c", "-o", obj, os.path.join(CSRC, u + ".cu")]
+        extra = os.environ.get("FSMSPEC_EXTRA_FLAGS", "").split()  # experiments only
+        cmd = [NVCC, *FLAGS, *extra, "-I", os.path.join(ROOT, "include"), "-c", "-o", obj, os.path.join(CSRC, u + ".cu")]
         res = subprocess.run(cmd, capture_output=True, text=True)
         return u, obj, cmd, res
 

@@ -455,7 +455,11 @@ struct RunSpec {
     uint32_t merge;
     uint64_t geom_len_bytes = 0;  // geometry as for a run of this many bytes (0 = len): tuning samples
     uint32_t force_T = 0, force_chunk = 0;  // multi-FSM groups: one geometry for every DFA
+    bool multi = false;                     // launched by the multi-FSM kernel (never split)
 };
+
+// Chunks per tile: a split kernel (split_kernel(var, K)) gives the CTA's last warp to the epilogue.
+static uint32_t tile_chunks(uint32_t T, bool split) { return split ? T - 32 : T; }
 
 static int variant_of(const fsm *f, int force, uint32_t k = 1)
 {
@@ -523,7 +527,9 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     if (r.force_T) T = r.force_T;
     if (r.force_chunk) chunk = r.force_chunk;
     if (r.merge == FSM_MERGE_SEQUENTIAL) T = std::min<uint32_t>(T, kThreads);
-    const uint64_t tile_bytes = (uint64_t)T * chunk;
+    const bool split = split_kernel(var, K) && !r.multi && r.merge == FSM_MERGE_PARALLEL;
+    if (split && T < 64) T = 64;  // at least one worker warp besides the epilogue warp
+    const uint64_t tile_bytes = (uint64_t)tile_chunks(T, split) * chunk;
     uint64_t ntiles64 = (len_bytes + tile_bytes - 1) / tile_bytes;
     if (ntiles64 == 0) ntiles64 = 1;
     if (ntiles64 > 0x7FFFFFFFull) return FSM_EINVAL;
@@ -567,13 +573,13 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
 
     if (var == VAR_HS) {
         // as many hot rows as fit next to this launch's scratch (227 KB per CTA)
-        const uint32_t scratch = Layout(T, K, 0).total;
+        const uint32_t scratch = Layout(T, K, 0, split).total;
         const uint32_t avail = scratch < 232448u ? 232448u - scratch : 0u;
         const uint32_t hot = std::min<uint32_t>(f->hot_rows, avail / 512);
         p.hot_rows = hot;
         p.table_bytes = hot * 512;
     }
-    const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes)).total;
+    const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes), split).total;
 
     if (p.lookback >= 32) {
         // a3 pre-pass: ranked look-back candidates per chunk (spec_kernel.cuh)
@@ -614,7 +620,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     f->last.chunks = (len_bytes + chunk - 1) / chunk;
     f->last.tiles = ntiles;
     f->last.chunk_bytes = chunk;
-    f->last.threads_per_tile = T;
+    f->last.threads_per_tile = tile_chunks(T, split);
     f->last.variant = var;
     f->last.k_slots = K;
     f->last.lookback_len = p.lookback;
@@ -1089,7 +1095,7 @@ extern "C" int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *inpu
         for (uint32_t n = 0; n < g.size() && rc == FSM_OK; n++) {
             fsm *f = fsms[g[n]];
             RunSpec r{nullptr, input, len, k[g[n]], false, 0, f->start_int, nullptr, f->d_result, var,
-                      FSM_MERGE_PARALLEL, 0, T, chunk};
+                      FSM_MERGE_PARALLEL, 0, T, chunk, true};
             Prepared pr;
             if ((rc = prepare_run(f, r, pr))) break;
             hp[base + n] = pr.p;

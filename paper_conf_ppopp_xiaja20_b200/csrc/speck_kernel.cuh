@@ -39,7 +39,10 @@ constexpr uint32_t kExtNone = 0xFFFFu;
 // caps them for large K.
 // (K = 2, 3 at 768 threads get 85 registers: the multi-chain prologue spills at 64; measured
 // +6 % over 1024 threads for (8, 2, k=2).)
-__host__ __device__ constexpr int max_threads(int K) { return K == 1 ? 1024 : K <= 3 ? 768 : K <= 6 ? 512 : 256; }
+#ifndef FSM_T1
+#define FSM_T1 1024
+#endif
+__host__ __device__ constexpr int max_threads(int K) { return K == 1 ? FSM_T1 : K <= 3 ? 768 : K <= 6 ? 512 : 256; }
 __host__ __device__ constexpr int min_blocks(int) { return 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
 
@@ -544,11 +547,38 @@ __device__ __forceinline__ bool chains_converged(const TB &tb, const uint32_t (&
 // Blocks [i, nblk) of 32 bytes with a 3-buffer rotation (2 blocks in flight, no register moves).
 // On entry x0 = block i, x1 = block i+1.  With CHECK, returns true as soon as the warp votes
 // that all chains coincide; x0/x1 then hold blocks i, i+1 for the continuation.
+#ifndef FSM_NBUF
+#define FSM_NBUF 3
+#endif
 template <int KK, bool CHECK, class TB>
 __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint64_t &i, uint64_t nblk, Bytes32 &x0,
                                            Bytes32 &x1, uint32_t (&cur)[KK], uint32_t (&acc)[KK],
                                            uint32_t (&accf)[KK])
 {
+#if FSM_NBUF == 2
+    // two buffers: block i+2 is requested after block i is consumed (16 registers of input in
+    // flight instead of 24; the freed registers let the table-row loads run ahead of their use)
+    while (i < nblk) {
+        process32<KK>(tb, x0, cur, acc, accf);
+        ++i;
+        if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
+            x0 = x1;
+            if (i + 1 < nblk) x1 = ldg_block(p, i + 1, nblk);
+            return true;
+        }
+        if (i >= nblk) break;
+        if (i + 1 < nblk) x0 = ldg_block(p, i + 1, nblk);
+        process32<KK>(tb, x1, cur, acc, accf);
+        ++i;
+        if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
+            if (i + 1 < nblk) x1 = ldg_block(p, i + 1, nblk);  // x0 already holds block i
+            return true;
+        }
+        if (i >= nblk) break;
+        if (i + 1 < nblk) x1 = ldg_block(p, i + 1, nblk);
+    }
+    return false;
+#else
     Bytes32 x2;
     while (i < nblk) {
         if (i + 2 < nblk) x2 = ldg_block(p, i + 2, nblk);
@@ -578,6 +608,7 @@ __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint6
         }
     }
     return false;
+#endif
 }
 
 // Alg. 3 over bytes [b, e) of the input: 32-byte blocks (one full sector per lane per
@@ -748,25 +779,62 @@ __device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eo
 }
 
 // ----------------------------------------------------------------- shared-memory layout ----
+// Split mode (dedicated epilogue warp): the tile state the epilogue reads (qe, qc, sj, ext) is
+// double-buffered -- buffer b at offset b * buf -- and there is no stash (re-execution and eager
+// completion read the chunk's first bytes from L2 instead).
 struct Layout {
-    uint32_t qe, qc, sj, ws, we, wc, wi, misc, stash, ext, total;
-    __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t start)
+    uint32_t qe, qc, sj, ws, we, wc, wi, misc, stash, ext, total, buf;
+    __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t start, bool split = false)
     {
         uint32_t o = start;
         qe = o;  o += T * K * 4;
         qc = o;  o += T * K * 4;
         sj = o;  o += T * K * 2;
         o = (o + 15) & ~15u;
+        if (split) {
+            ext = o; o += T * kExt * 4;
+            buf = o - qe;
+            o += buf;
+            stash = 0;
+        }
         ws = o;  o += 32 * K * 4;
         we = o;  o += 32 * K * 4;
         wc = o;  o += 32 * K * 4;
         wi = o;  o += 32 * 4;
         misc = o; o += 16;
-        stash = o; o += T * 32;
-        ext = o; o += T * kExt * 4;
+        if (!split) {
+            stash = o; o += T * 32;
+            ext = o; o += T * kExt * 4;
+            buf = 0;
+        }
         total = o;
     }
 };
+
+// Named barriers of the split kernel: 1 = worker warps; 2, 3 = tile state of buffer 0 / 1 handed to
+// the epilogue warp; 4, 5 = buffer 0 / 1 free again.
+__device__ __forceinline__ void named_sync(uint32_t id, uint32_t n)
+{
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void named_arrive(uint32_t id, uint32_t n)
+{
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+// Which fused kernels run split (measured on B200, 4 GiB inputs, split vs unsplit): the CL variant
+// (HTML, k = 1: +13 %, its serial re-executions dominate the epilogue) and the multi-chain kernels
+// of the shared-memory variants (P4 / P8 / B, K >= 2: +6..15 %).  K = 1 kernels of P8 / B / G / HS
+// lose more from the missing 32nd worker warp and stash than they gain (-4..-8 %): unsplit.
+// FSM_SPLIT: 2 = this policy (default), 1 = always, 0 = never (experiments).
+#ifndef FSM_SPLIT
+#define FSM_SPLIT 2
+#endif
+__host__ __device__ constexpr bool split_kernel(int var, int K)
+{
+    return FSM_SPLIT == 1 ? true
+         : FSM_SPLIT == 0 ? false
+         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 4 || var == 2) /* P4 P8 H8 B */ && K >= 2));
+}
 
 // Per-tile context used by re-execution and the epilogue.
 struct TileCtx {
@@ -850,7 +918,7 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
                     cyc = cy[l];
                 }
         };
-        if (t.aligned && e - b >= 32) {
+        if (t.stash && t.aligned && e - b >= 32) {
             // the chunk's first 32 bytes were stashed in smem by its owner during the local phase:
             // the usual early exit never touches global memory
 #pragma unroll 1
@@ -907,6 +975,242 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
     }
 }
 
+// a7-a9 for one tile, run by one full warp once the tile's suffix mappings Qe/Qc (keyed on the
+// chunks' speculated starts Sj) are in shared memory: pre-resolution of the tile aggregate's broken
+// slots (R5), publication of A, decoupled look-back, own inclusive prefix P, and the result.
+template <int K, class TB>
+__device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uint32_t tile, uint64_t tile_base,
+                                              uint32_t nch_max, uint32_t *Qe, uint32_t *Qc, const uint16_t *Sj,
+                                              const uint32_t *stash, const uint32_t *Ext, uint32_t start_state,
+                                              unsigned long long start_count, uint32_t ksel)
+{
+    const int lane = threadIdx.x & 31;
+    TileCtx t;
+    t.in = p.in;
+    t.len = p.len;
+    t.tile_base = tile_base;
+    t.chunk = p.chunk;
+    {
+        const uint64_t rem = p.len > tile_base ? p.len - tile_base : 0;
+        const uint64_t nch = (rem + p.chunk - 1) / p.chunk;
+        t.nch = (uint32_t)(nch < 1 ? 1 : (nch > nch_max ? nch_max : nch));
+    }
+    t.aligned = p.aligned != 0;
+    t.Qe = Qe;
+    t.Qc = Qc;
+    t.Sj = Sj;
+    t.stash = stash;
+    t.ext = Ext;
+    t.stats = p.stats;
+
+    // a8 (tile candidates): resolve the broken slots of the tile aggregate Q_0 so that the
+    // published aggregate is complete on every speculated tile start.
+    if (lane < K) {
+        const uint32_t x = Qe[lane];
+        if ((x >> 16) < ABSENT) {
+            uint32_t st, n;
+            resolve<K>(tb, t, x & 0xFFFFu, x >> 16, Qc[lane], st, n);
+            Qe[lane] = st | (COMPLETE << 16);
+            Qc[lane] = n;
+        }
+    }
+    __syncwarp();
+
+    // a7: publish the aggregate A_b (slot = {start, end, count})
+    TileDesc *D = p.desc + tile;
+    if (lane < K) {
+        const uint32_t sv = Sj[lane];
+        D->aslot[lane] = make_uint4(sv == 0xFFFFu ? NOSTATE : sv, Qe[lane] & 0xFFFFu, Qc[lane], 0u);
+    }
+    __threadfence();
+    __syncwarp();
+    const uint32_t ep = p.epoch << 2;
+    if (lane == 0) st_release(&D->flag, ep | ST_A);
+
+    // a7: decoupled look-back -> exclusive prefix E (lane s holds shard slot s).
+    // (1) walk back 32 descriptors at a time to the nearest inclusive prefix P_m.
+    uint32_t Es = 0;
+    unsigned long long Ec = 0;
+    bool Ev = false;
+    int64_t m;
+    {
+        int64_t base = (int64_t)tile - 1;
+        for (;;) {
+            const int64_t tt = base - lane;
+            uint32_t st = ST_P;
+            if (tt >= 0) {
+                const uint32_t f = ld_acquire(&p.desc[tt].flag);
+                st = (f & ~3u) == ep ? (f & 3u) : (uint32_t)ST_X;
+            }
+            const unsigned pm = __ballot_sync(0xFFFFFFFFu, st == ST_P);
+            const unsigned xm = __ballot_sync(0xFFFFFFFFu, st == ST_X);
+            const int fp = pm ? __ffs(pm) - 1 : 32;
+            const unsigned before = fp >= 32 ? 0xFFFFFFFFu : ((1u << fp) - 1u);
+            if (xm & before) {
+                __nanosleep(64);
+                continue;
+            }
+            if (fp < 32) {
+                m = base - fp;
+                break;
+            }
+            base -= 32;
+        }
+    }
+    auto load_P = [&](int64_t tt) {
+        const TileDesc *Dt = p.desc + tt;
+        while (ld_acquire(&Dt->flag) != (ep | ST_P)) __nanosleep(64);
+        const uint32_t pmask = __ldcg(&Dt->pmask);
+        Ev = lane < KMAX && ((pmask >> lane) & 1u);
+        if (lane < KMAX) {
+            Es = __ldcg(&Dt->pstate[lane]);
+            Ec = __ldcg(&Dt->pcnt[lane]);
+        }
+    };
+    if (m < 0) {
+        if (!p.keyed) {
+            Ev = lane == 0;
+            Es = start_state;
+            Ec = start_count;
+        } else {
+            const uint32_t c = p.halo_byte;
+            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
+            Ev = (uint32_t)lane < ni;
+            Es = Ev ? (uint32_t)__ldg(p.lb + c * KMAX + lane) : 0u;
+            Ec = 0;
+        }
+    } else {
+        load_P(m);
+    }
+    // (2) apply the aggregates A_{m+1} .. A_{b-1}, 32 per step: every lane loads one tile's
+    // aggregate in parallel, a warp suffix scan composes the 32 mappings (the same operator as
+    // the chunk merge), and the composed window is applied to E.  A slot that breaks inside the
+    // window hit a tile-boundary miss there: take that tile's P and continue after it.
+    for (int64_t nx = m + 1; nx < (int64_t)tile;) {
+        const int64_t tt = nx + lane;
+        uint32_t S2[K], e2[K], c2[K];
+        bool id2 = tt >= (int64_t)tile;
+        if (!id2) {
+            const TileDesc *Dt = p.desc + tt;
+            while ((ld_acquire(&Dt->flag) & ~3u) != ep) __nanosleep(32);
+#pragma unroll
+            for (int l = 0; l < K; l++) {
+                const uint4 v = __ldcg(&Dt->aslot[l]);
+                S2[l] = v.x;
+                e2[l] = v.x == NOSTATE ? (ABSENT << 16) : (v.y | (COMPLETE << 16));
+                c2[l] = v.z;
+            }
+        } else {
+#pragma unroll
+            for (int l = 0; l < K; l++) S2[l] = NOSTATE, e2[l] = ABSENT << 16, c2[l] = 0;
+        }
+        warp_suffix_scan<K>(S2, e2, c2, id2, 0, 1);
+        int brk = 32;
+        {
+            uint32_t ne = 0, nc = 0;
+            bool found = false;
+#pragma unroll
+            for (int l = 0; l < K; l++) {
+                const uint32_t sl = __shfl_sync(0xFFFFFFFFu, S2[l], 0);
+                const uint32_t el = __shfl_sync(0xFFFFFFFFu, e2[l], 0);
+                const uint32_t cl = __shfl_sync(0xFFFFFFFFu, c2[l], 0);
+                if (Ev && sl == Es) {
+                    ne = el;
+                    nc = cl;
+                    found = true;
+                }
+            }
+            if (Ev) {
+                if (!found) brk = 0;
+                else if ((ne >> 16) != COMPLETE) brk = (int)(ne >> 16);
+                else {
+                    Es = ne & 0xFFFFu;
+                    Ec += nc;
+                }
+            }
+        }
+        const int mb = __reduce_min_sync(0xFFFFFFFFu, brk);
+        if (mb < 32) {
+            load_P(nx + mb);  // E := P of the tile where a slot broke (it resolves its own miss)
+            nx = nx + mb + 1;
+        } else {
+            nx += 32;
+        }
+    }
+
+    // own inclusive prefix P_b = E then A_b; a tile-boundary miss resolves through chunk 0.
+    uint32_t Ps = 0;
+    unsigned long long Pc = 0;
+    if (Ev) {
+        bool hit = false;
+#pragma unroll
+        for (int l = 0; l < K; l++)
+            if (!hit && Sj[l] == Es) {
+                Ps = Qe[l] & 0xFFFFu;
+                Pc = Ec + Qc[l];
+                hit = true;
+            }
+        if (!hit) {
+            uint32_t st, n;
+            resolve<K>(tb, t, Es, 0, 0, st, n);
+            Ps = st;
+            Pc = Ec + n;
+            atomicAdd(&p.stats->boundary_misses, 1ull);
+        }
+    }
+    const unsigned vmask = __ballot_sync(0xFFFFFFFFu, Ev);
+    if (lane < KMAX) {
+        D->pstate[lane] = Ps;
+        D->pcnt[lane] = Pc;
+    }
+    if (lane == 0) D->pmask = vmask;
+    __threadfence();
+    __syncwarp();
+    if (lane == 0) st_release(&D->flag, ep | ST_P);
+
+    // a9: the last tile writes the result (bit-mode tail applied here)
+    if (tile == p.ntiles - 1) {
+        uint32_t x = Ps;
+        unsigned long long cc = Pc;
+        if (Ev && p.tail_bits) {
+            const uint32_t tail_byte = __ldg(p.in + p.len);
+            for (uint32_t i = 0; i < p.tail_bits; i++) {
+                const uint32_t bit = (tail_byte >> (7 - i)) & 1u;
+                const uint32_t en = __ldg(p.bittab + x * 2 + bit);
+                x = en & 0xFFFFu;
+                cc += en >> 16;
+            }
+        }
+        DevResult *R = p.result;
+        if (!p.keyed) {
+            if (lane == 0) {
+                R->final_state = x;  // internal id (chains pieces on the device)
+                R->status = 0;
+                R->count = cc;
+                if (p.user_out) {
+                    p.user_out[0] = p.inv ? __ldg(p.inv + x) : x;
+                    p.user_out[1] = 0;
+                    p.user_out[2] = (uint32_t)cc;
+                    p.user_out[3] = (uint32_t)(cc >> 32);
+                }
+            }
+        } else {
+            const uint32_t c = p.halo_byte;
+            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
+            if (lane < KMAX) {
+                R->start[lane] = (uint32_t)lane < ni ? (uint32_t)__ldg(p.lb + c * KMAX + lane) : NOSTATE;
+                R->end[lane] = x;
+                R->mcount[lane] = cc;
+            }
+            if (lane == 0) {
+                R->valid_mask = vmask;
+                R->k = ksel;
+                R->status = 0;
+            }
+        }
+    }
+}
+
 // ------------------------------------------------------------------------------- the kernel --
 // The body serves two kernels.  speck_kernel: one DFA, parameters in the kernel parameter space.
 // speck_multi_kernel (NEXT-4, many FSMs over one resident input): M DFAs of the same
@@ -915,18 +1219,24 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
 // time and the tile is read from HBM once and from L2 M - 1 times.  Each DFA keeps its own
 // descriptors (its own decoupled look-back), result and counters (pm[d]); a CTA reloads the table
 // image into shared memory when its ticket switches DFA.
-template <int K, int VAR, bool MULTI>
+// SPLIT (speck_kernel with FSM_SPLIT): the last warp of the CTA is a dedicated epilogue warp; the
+// other warps (T - 32 chunks per tile) hand each tile's state over in one of two buffers and go
+// straight on to the next tile, so the serial epilogue (pre-resolution re-executions, look-back)
+// overlaps the next tile's local phase instead of idling the SM at a barrier.
+template <int K, int VAR, bool MULTI, bool SPLIT = false>
 __device__ __forceinline__ void speck_body(const Params &p0, const Params *__restrict__ pm, uint32_t M)
 {
+    static_assert(!(MULTI && SPLIT), "multi-FSM runs use the unsplit body");
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];  // no static shared memory: see kSmemWindowBase
 
     const uint32_t T = blockDim.x;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = T >> 5;
+    const uint32_t TW = SPLIT ? T - 32 : T;  // chunks per tile
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = TW >> 5;
     const uint32_t j = threadIdx.x;
 
     // MULTI: p0.table_bytes is the group's largest table image, so one layout serves every DFA
-    const Layout L(T, K, scratch_offset(VAR, p0.table_bytes));
+    const Layout L(T, K, scratch_offset(VAR, p0.table_bytes), SPLIT);
     check_smem_window(VAR, L.total);
     TB tb;
     if (!MULTI) tb.setup(smem, p0.table, p0.n_states, kconst(p0));
@@ -941,13 +1251,52 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
     uint32_t *Ext = reinterpret_cast<uint32_t *>(smem + L.ext);
     const uint32_t ntickets = MULTI ? p0.ntiles * M : p0.ntiles;
     uint32_t loaded = 0xFFFFFFFFu;  // MULTI: DFA whose table image is in shared memory
+    uint32_t *s_tiles = &s_tile;    // SPLIT: one ticket slot per buffer
 
-    for (;;) {
-        __syncthreads();  // smem reuse across tiles; also orders the table setup
-        if (threadIdx.x == 0) s_tile = atomicAdd(p0.ticket, 1u) - p0.ticket_base;
-        __syncthreads();
-        const uint32_t ticket = s_tile;
-        if (ticket >= ntickets) break;
+    if (SPLIT && warp == W) {
+        // ---- the epilogue warp: tiles in ticket order, buffers alternating
+        __syncthreads();  // table setup done
+        const uint32_t start_state = p0.start_dev ? p0.start_dev->final_state : p0.start_state;
+        const unsigned long long start_count = p0.start_dev ? p0.start_dev->count : 0ull;
+        named_arrive(4, T);
+        named_arrive(5, T);
+        for (uint32_t it = 0;; it++) {
+            const uint32_t bb = it & 1u;
+            named_sync(2 + bb, T);
+            const uint32_t tile = s_tiles[bb];
+            if (tile >= p0.ntiles) break;
+            const uint32_t o = bb * L.buf;
+            tile_epilogue<K>(tb, p0, tile, (uint64_t)tile * TW * p0.chunk, TW,
+                             reinterpret_cast<uint32_t *>(smem + L.qe + o), reinterpret_cast<uint32_t *>(smem + L.qc + o),
+                             reinterpret_cast<const uint16_t *>(smem + L.sj + o), nullptr,
+                             reinterpret_cast<const uint32_t *>(smem + L.ext + o), start_state, start_count, p0.k);
+            __syncwarp();
+            named_arrive(4 + bb, T);
+        }
+        return;
+    }
+    if (SPLIT) __syncthreads();  // table setup done (matches the epilogue warp's)
+
+    for (uint32_t it = 0;; it++) {
+        const uint32_t bb = SPLIT ? (it & 1u) : 0u;
+        if (SPLIT) {
+            named_sync(4 + bb, T);  // buffer bb free: the epilogue is done with tile it - 2
+            if (threadIdx.x == 0) s_tiles[bb] = atomicAdd(p0.ticket, 1u) - p0.ticket_base;
+            named_sync(1, TW);
+            Qe = reinterpret_cast<uint32_t *>(smem + L.qe + bb * L.buf);
+            Qc = reinterpret_cast<uint32_t *>(smem + L.qc + bb * L.buf);
+            Sj = reinterpret_cast<uint16_t *>(smem + L.sj + bb * L.buf);
+            Ext = reinterpret_cast<uint32_t *>(smem + L.ext + bb * L.buf);
+        } else {
+            __syncthreads();  // smem reuse across tiles; also orders the table setup
+            if (threadIdx.x == 0) s_tile = atomicAdd(p0.ticket, 1u) - p0.ticket_base;
+            __syncthreads();
+        }
+        const uint32_t ticket = s_tiles[bb];
+        if (ticket >= ntickets) {
+            if (SPLIT) named_arrive(2 + bb, T);  // tells the epilogue warp to stop
+            break;
+        }
         const uint32_t dfa = MULTI ? ticket % M : 0u;
         const uint32_t tile = MULTI ? ticket / M : ticket;
         const Params &p = MULTI ? pm[dfa] : p0;
@@ -960,7 +1309,7 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
         const unsigned long long start_count = p.start_dev ? p.start_dev->count : 0ull;
         const uint32_t ksel = p.k;
 
-        const uint64_t tile_base = (uint64_t)tile * T * p.chunk;
+        const uint64_t tile_base = (uint64_t)tile * TW * p.chunk;
         const uint64_t b = tile_base + (uint64_t)j * p.chunk;
         const bool first_chunk = tile == 0 && j == 0;
         const bool empty = b >= p.len && !first_chunk;
@@ -981,9 +1330,8 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
             acc[s] = 0;
             accf[s] = 0;
         }
-        if (!empty && e > b)
-            local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf,
-                           reinterpret_cast<uint32_t *>(smem + L.stash) + j * 8);
+        uint32_t *const stash_j = SPLIT ? nullptr : reinterpret_cast<uint32_t *>(smem + L.stash) + j * 8;
+        if (!empty && e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf, stash_j);
         uint32_t eob[K], cnt[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
@@ -999,7 +1347,6 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
 #pragma unroll
             for (int q = 0; q < kExt; q++) ent[q] = kExtNone;
             if (p.eager_window && p.aligned && !empty && e - b >= 32 && Xc[0] != NOSTATE) {
-                const uint32_t *st32 = reinterpret_cast<const uint32_t *>(smem + L.stash) + j * 8;
                 uint32_t y[K], cy[K], u[kExt], cu[kExt];
                 bool live[kExt];
 #pragma unroll
@@ -1020,9 +1367,9 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
 #pragma unroll 1
                 for (uint32_t blk = 0; blk < wlen && nlive > 0; blk += 32) {
                     Bytes32 xb;
-                    if (blk == 0) {
+                    if (blk == 0 && stash_j) {
 #pragma unroll
-                        for (int q = 0; q < 8; q++) xb.w[q] = st32[q];
+                        for (int q = 0; q < 8; q++) xb.w[q] = stash_j[q];
                     } else {
                         xb = ldg256(p.in + b + blk);
                     }
@@ -1070,7 +1417,7 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
             }
             wI[warp] = ident;
         }
-        __syncthreads();
+        if (SPLIT) named_sync(1, TW); else __syncthreads();
         if (warp == 0) {
             uint32_t S2[K], e2[K], c2[K];
             bool id2 = true;
@@ -1096,7 +1443,7 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
                 }
             }
         }
-        __syncthreads();
+        if (SPLIT) named_sync(1, TW); else __syncthreads();
         if (warp + 1 < W && !ident && wI[warp + 1] == 0) {
             uint32_t Sr[K], er[K], cr[K];
 #pragma unroll
@@ -1113,6 +1460,10 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
             Qc[j * K + s] = cnt[s];
             Sj[j * K + s] = (uint16_t)(S[s] == NOSTATE ? 0xFFFFu : S[s]);
         }
+        if (SPLIT) {
+            named_arrive(2 + bb, T);  // hand the tile over to the epilogue warp
+            continue;
+        }
         __syncthreads();
 
 #ifdef FSM_PHASE_TIMING
@@ -1122,246 +1473,15 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
         if (warp != 0) continue;
 
         // ================= warp 0: tile epilogue (pre-resolution, look-back, publication) =====
-        TileCtx t;
-        t.in = p.in;
-        t.len = p.len;
-        t.tile_base = tile_base;
-        t.chunk = p.chunk;
-        {
-            const uint64_t rem = p.len > tile_base ? p.len - tile_base : 0;
-            const uint64_t nch = (rem + p.chunk - 1) / p.chunk;
-            t.nch = (uint32_t)(nch < 1 ? 1 : (nch > T ? T : nch));
-        }
-        t.aligned = p.aligned != 0;
-        t.Qe = Qe;
-        t.Qc = Qc;
-        t.Sj = Sj;
-        t.stash = reinterpret_cast<const uint32_t *>(smem + L.stash);
-        t.ext = Ext;
-        t.stats = p.stats;
-
-        // a8 (tile candidates): resolve the broken slots of the tile aggregate Q_0 so that the
-        // published aggregate is complete on every speculated tile start.
-        if (lane < K) {
-            const uint32_t x = Qe[lane];
-            if ((x >> 16) < ABSENT) {
-                uint32_t st, n;
-                resolve<K>(tb, t, x & 0xFFFFu, x >> 16, Qc[lane], st, n);
-                Qe[lane] = st | (COMPLETE << 16);
-                Qc[lane] = n;
-            }
-        }
-        __syncwarp();
-
-        // a7: publish the aggregate A_b (slot = {start, end, count})
-        TileDesc *D = p.desc + tile;
-        if (lane < K) {
-            const uint32_t sv = Sj[lane];
-            D->aslot[lane] = make_uint4(sv == 0xFFFFu ? NOSTATE : sv, Qe[lane] & 0xFFFFu, Qc[lane], 0u);
-        }
-        __threadfence();
-        __syncwarp();
-        const uint32_t ep = p.epoch << 2;
-        if (lane == 0) st_release(&D->flag, ep | ST_A);
-
-        // a7: decoupled look-back -> exclusive prefix E (lane s holds shard slot s).
-        // (1) walk back 32 descriptors at a time to the nearest inclusive prefix P_m.
-        uint32_t Es = 0;
-        unsigned long long Ec = 0;
-        bool Ev = false;
-        int64_t m;
-        {
-            int64_t base = (int64_t)tile - 1;
-            for (;;) {
-                const int64_t tt = base - lane;
-                uint32_t st = ST_P;
-                if (tt >= 0) {
-                    const uint32_t f = ld_acquire(&p.desc[tt].flag);
-                    st = (f & ~3u) == ep ? (f & 3u) : (uint32_t)ST_X;
-                }
-                const unsigned pm = __ballot_sync(0xFFFFFFFFu, st == ST_P);
-                const unsigned xm = __ballot_sync(0xFFFFFFFFu, st == ST_X);
-                const int fp = pm ? __ffs(pm) - 1 : 32;
-                const unsigned before = fp >= 32 ? 0xFFFFFFFFu : ((1u << fp) - 1u);
-                if (xm & before) {
-                    __nanosleep(64);
-                    continue;
-                }
-                if (fp < 32) {
-                    m = base - fp;
-                    break;
-                }
-                base -= 32;
-            }
-        }
-        auto load_P = [&](int64_t tt) {
-            const TileDesc *Dt = p.desc + tt;
-            while (ld_acquire(&Dt->flag) != (ep | ST_P)) __nanosleep(64);
-            const uint32_t pmask = __ldcg(&Dt->pmask);
-            Ev = lane < KMAX && ((pmask >> lane) & 1u);
-            if (lane < KMAX) {
-                Es = __ldcg(&Dt->pstate[lane]);
-                Ec = __ldcg(&Dt->pcnt[lane]);
-            }
-        };
-        if (m < 0) {
-            if (!p.keyed) {
-                Ev = lane == 0;
-                Es = start_state;
-                Ec = start_count;
-            } else {
-                const uint32_t c = p.halo_byte;
-                const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
-                Ev = (uint32_t)lane < ni;
-                Es = Ev ? (uint32_t)__ldg(p.lb + c * KMAX + lane) : 0u;
-                Ec = 0;
-            }
-        } else {
-            load_P(m);
-        }
-        // (2) apply the aggregates A_{m+1} .. A_{b-1}, 32 per step: every lane loads one tile's
-        // aggregate in parallel, a warp suffix scan composes the 32 mappings (the same operator as
-        // the chunk merge), and the composed window is applied to E.  A slot that breaks inside the
-        // window hit a tile-boundary miss there: take that tile's P and continue after it.
-        for (int64_t nx = m + 1; nx < (int64_t)tile;) {
-            const int64_t tt = nx + lane;
-            uint32_t S2[K], e2[K], c2[K];
-            bool id2 = tt >= (int64_t)tile;
-            if (!id2) {
-                const TileDesc *Dt = p.desc + tt;
-                while ((ld_acquire(&Dt->flag) & ~3u) != ep) __nanosleep(32);
-#pragma unroll
-                for (int l = 0; l < K; l++) {
-                    const uint4 v = __ldcg(&Dt->aslot[l]);
-                    S2[l] = v.x;
-                    e2[l] = v.x == NOSTATE ? (ABSENT << 16) : (v.y | (COMPLETE << 16));
-                    c2[l] = v.z;
-                }
-            } else {
-#pragma unroll
-                for (int l = 0; l < K; l++) S2[l] = NOSTATE, e2[l] = ABSENT << 16, c2[l] = 0;
-            }
-            warp_suffix_scan<K>(S2, e2, c2, id2, 0, 1);
-            int brk = 32;
-            {
-                uint32_t ne = 0, nc = 0;
-                bool found = false;
-#pragma unroll
-                for (int l = 0; l < K; l++) {
-                    const uint32_t sl = __shfl_sync(0xFFFFFFFFu, S2[l], 0);
-                    const uint32_t el = __shfl_sync(0xFFFFFFFFu, e2[l], 0);
-                    const uint32_t cl = __shfl_sync(0xFFFFFFFFu, c2[l], 0);
-                    if (Ev && sl == Es) {
-                        ne = el;
-                        nc = cl;
-                        found = true;
-                    }
-                }
-                if (Ev) {
-                    if (!found) brk = 0;
-                    else if ((ne >> 16) != COMPLETE) brk = (int)(ne >> 16);
-                    else {
-                        Es = ne & 0xFFFFu;
-                        Ec += nc;
-                    }
-                }
-            }
-            const int mb = __reduce_min_sync(0xFFFFFFFFu, brk);
-            if (mb < 32) {
-                load_P(nx + mb);  // E := P of the tile where a slot broke (it resolves its own miss)
-                nx = nx + mb + 1;
-            } else {
-                nx += 32;
-            }
-        }
-
-        // own inclusive prefix P_b = E then A_b; a tile-boundary miss resolves through chunk 0.
-        uint32_t Ps = 0;
-        unsigned long long Pc = 0;
-        if (Ev) {
-            bool hit = false;
-#pragma unroll
-            for (int l = 0; l < K; l++)
-                if (!hit && Sj[l] == Es) {
-                    Ps = Qe[l] & 0xFFFFu;
-                    Pc = Ec + Qc[l];
-                    hit = true;
-                }
-            if (!hit) {
-                uint32_t st, n;
-                resolve<K>(tb, t, Es, 0, 0, st, n);
-                Ps = st;
-                Pc = Ec + n;
-                atomicAdd(&p.stats->boundary_misses, 1ull);
-            }
-        }
-        const unsigned vmask = __ballot_sync(0xFFFFFFFFu, Ev);
-        if (lane < KMAX) {
-            D->pstate[lane] = Ps;
-            D->pcnt[lane] = Pc;
-        }
-        if (lane == 0) D->pmask = vmask;
-        __threadfence();
-        __syncwarp();
-        if (lane == 0) st_release(&D->flag, ep | ST_P);
-
-#ifdef FSM_PHASE_TIMING
-        if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 42, (unsigned long long)(clock64() - t_scan1));
-        if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 43, 1ull);
-        if (threadIdx.x == 0 && tile == p.ntiles - 1) {
-            unsigned long long *q = reinterpret_cast<unsigned long long *>(p.result) + 40;
-            printf("PHASES local(sum over threads)=%llu scan+merge(t0)=%llu epilogue(t0)=%llu tiles=%llu T=%u\n", q[0], q[1], q[2], q[3], T);
-            q[0] = q[1] = q[2] = q[3] = 0;
-        }
-#endif
-        // a9: the last tile writes the result (bit-mode tail applied here)
-        if (tile == p.ntiles - 1) {
-            uint32_t x = Ps;
-            unsigned long long cc = Pc;
-            if (Ev && p.tail_bits) {
-                const uint32_t tail_byte = __ldg(p.in + p.len);
-                for (uint32_t i = 0; i < p.tail_bits; i++) {
-                    const uint32_t bit = (tail_byte >> (7 - i)) & 1u;
-                    const uint32_t en = __ldg(p.bittab + x * 2 + bit);
-                    x = en & 0xFFFFu;
-                    cc += en >> 16;
-                }
-            }
-            DevResult *R = p.result;
-            if (!p.keyed) {
-                if (lane == 0) {
-                    R->final_state = x;  // internal id (chains pieces on the device)
-                    R->status = 0;
-                    R->count = cc;
-                    if (p.user_out) {
-                        p.user_out[0] = p.inv ? __ldg(p.inv + x) : x;
-                        p.user_out[1] = 0;
-                        p.user_out[2] = (uint32_t)cc;
-                        p.user_out[3] = (uint32_t)(cc >> 32);
-                    }
-                }
-            } else {
-                const uint32_t c = p.halo_byte;
-                const uint32_t ni = min((uint32_t)__ldg(p.nimg + c), ksel);
-                if (lane < KMAX) {
-                    R->start[lane] = (uint32_t)lane < ni ? (uint32_t)__ldg(p.lb + c * KMAX + lane) : NOSTATE;
-                    R->end[lane] = x;
-                    R->mcount[lane] = cc;
-                }
-                if (lane == 0) {
-                    R->valid_mask = vmask;
-                    R->k = ksel;
-                    R->status = 0;
-                }
-            }
-        }
+        tile_epilogue<K>(tb, p, tile, tile_base, TW, Qe, Qc, Sj, reinterpret_cast<const uint32_t *>(smem + L.stash), Ext,
+                         start_state, start_count, ksel);
     }
 }
 
 template <int K, int VAR>
 __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Params p)
 {
-    speck_body<K, VAR, false>(p, nullptr, 1);
+    speck_body<K, VAR, false, split_kernel(VAR, K)>(p, nullptr, 1);
 }
 
 template <int K, int VAR>

@@ -361,7 +361,7 @@ def main():
     peak = float(peaks.get("hbm_gbs", 6650.0))
     traffic = None
     if args.config == "c5" and args.n_states == 8 and args.m == 2 and args.k == 2:
-        traffic = round(1.031 * n)   # per launch, from the committed ncu capture of this config
+        traffic = round(1.037 * n)   # per launch: dram read+write / input bytes of the committed ncu capture
     line = {
         "metric": METRIC, "value": round(gbs, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(step_s * 1e3, 4), "higher_is_better": True,
@@ -370,7 +370,7 @@ def main():
         "roofline": {"bound": "hbm", "achieved": round(n / step_s / 1e9, 3) if world == 1 else round(gbs / world, 3),
                      "peak": peak, "unit": "GB/s", "frac": round((n / step_s / 1e9) / peak, 4),
                      "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback"},
-        "traffic_note": "ncu --set full (profiles/r01_ncu_c5_n8m2k2_8GiB.txt): dram read+write = 1.031 x input bytes",
+        "traffic_note": "ncu --set full (profiles/r01_ncu_c5_n8m2k2_8GiB.txt): dram read+write = 1.037 x input bytes (8.881 GB read + 0.030 GB written for 8 GiB)",
         "clocks": clk.summary(),
         "gpu_launches": args.steps,  # one fused kernel per step (plus a fix-up kernel per miss round for N > 1)
         "result": {"final_state": final[0], "accept_count": final[1]},

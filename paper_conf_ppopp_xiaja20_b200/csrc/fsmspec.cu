@@ -39,7 +39,7 @@ typedef void (*MultiFn)(Params, const Params *, uint32_t);
 // Kernel instantiations live in one translation unit per table variant (kernels_*.cu, compiled in
 // parallel); each exports these accessors.
 #define FSM_DECLARE_VARIANT(NAME)                                   \
-    KernelFn get_kernel_##NAME(int K);                              \
+    KernelFn get_kernel_##NAME(int K, bool split);                  \
     MultiFn get_multi_##NAME(int K);                                \
     FixFn get_fix_##NAME();                                         \
     void get_seq_##NAME(int K, SeqLocalFn &l, SeqWalkFn &w);       \
@@ -52,16 +52,16 @@ FSM_DECLARE_VARIANT(g)
 FSM_DECLARE_VARIANT(hs)
 FSM_DECLARE_VARIANT(cl)
 
-static KernelFn get_kernel(int var, int K)
+static KernelFn get_kernel(int var, int K, bool split)
 {
     switch (var) {
-    case VAR_P4: return get_kernel_p4(K);
-    case VAR_P8: return get_kernel_p8(K);
-    case VAR_H8: return get_kernel_h8(K);
-    case VAR_HS: return get_kernel_hs(K);
-    case VAR_CL: return get_kernel_cl(K);
-    case VAR_B: return get_kernel_b(K);
-    default: return get_kernel_g(K);
+    case VAR_P4: return get_kernel_p4(K, split);
+    case VAR_P8: return get_kernel_p8(K, split);
+    case VAR_H8: return get_kernel_h8(K, split);
+    case VAR_HS: return get_kernel_hs(K, split);
+    case VAR_CL: return get_kernel_cl(K, split);
+    case VAR_B: return get_kernel_b(K, split);
+    default: return get_kernel_g(K, split);
     }
 }
 static MultiFn get_multi(int var, int K)
@@ -460,6 +460,7 @@ struct RunSpec {
 
 // Chunks per tile: a split kernel (split_kernel(var, K)) gives the CTA's last warp to the epilogue.
 static uint32_t tile_chunks(uint32_t T, bool split) { return split ? T - 32 : T; }
+constexpr uint32_t kMaxSmem = 232448u;  // dynamic shared memory per CTA on sm_100 (227 KiB)
 
 static int variant_of(const fsm *f, int force, uint32_t k = 1)
 {
@@ -514,6 +515,7 @@ struct Prepared {
     int var, K;
     uint32_t T;
     size_t smem;
+    bool split;
 };
 
 static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
@@ -527,8 +529,12 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     if (r.force_T) T = r.force_T;
     if (r.force_chunk) chunk = r.force_chunk;
     if (r.merge == FSM_MERGE_SEQUENTIAL) T = std::min<uint32_t>(T, kThreads);
-    const bool split = split_kernel(var, K) && !r.multi && r.merge == FSM_MERGE_PARALLEL;
-    if (split && T < 64) T = 64;  // at least one worker warp besides the epilogue warp
+    if (split_kernel(var, K) && T < 64) T = 64;  // at least one worker warp besides the epilogue warp
+    bool split = split_kernel(var, K) && !r.multi && r.merge == FSM_MERGE_PARALLEL;
+    if (split) {  // the double-buffered layout must fit next to the table (HS sizes its hot rows after)
+        const uint32_t tb = var == VAR_HS ? 0u : f->img_bytes[var];
+        split = Layout(T, K, scratch_offset(var, tb), true).total <= kMaxSmem;
+    }
     const uint64_t tile_bytes = (uint64_t)tile_chunks(T, split) * chunk;
     uint64_t ntiles64 = (len_bytes + tile_bytes - 1) / tile_bytes;
     if (ntiles64 == 0) ntiles64 = 1;
@@ -574,7 +580,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     if (var == VAR_HS) {
         // as many hot rows as fit next to this launch's scratch (227 KB per CTA)
         const uint32_t scratch = Layout(T, K, 0, split).total;
-        const uint32_t avail = scratch < 232448u ? 232448u - scratch : 0u;
+        const uint32_t avail = scratch < kMaxSmem ? kMaxSmem - scratch : 0u;
         const uint32_t hot = std::min<uint32_t>(f->hot_rows, avail / 512);
         p.hot_rows = hot;
         p.table_bytes = hot * 512;
@@ -611,6 +617,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     out.K = K;
     out.T = T;
     out.smem = smem;
+    out.split = split;
     if (r.merge == FSM_MERGE_SEQUENTIAL) return FSM_OK;
     if ((rc = ensure_desc(f, ntiles))) return rc;
     out.p.desc = f->d_desc;
@@ -641,7 +648,7 @@ static int launch_run(fsm *f, const RunSpec &r)
         return launch_seq(f, p, var, K, T);
     }
 
-    KernelFn fn = get_kernel(var, K);
+    KernelFn fn = get_kernel(var, K, pr.split);
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)T, smem));

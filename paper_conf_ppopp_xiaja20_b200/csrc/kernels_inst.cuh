@@ -17,17 +17,26 @@ typedef void (*MultiFn)(Params, const Params *, uint32_t);
 #define FSM_CAT2(a, b) a##b
 #define FSM_CAT(a, b) FSM_CAT2(a, b)
 
-KernelFn FSM_CAT(get_kernel_, FSM_VAR_NAME)(int K)
+template <int K>
+static KernelFn pick(bool split)
+{
+    if constexpr (split_kernel(FSM_VAR, K)) {
+        if (split) return speck_kernel<K, FSM_VAR, true>;
+    }
+    return speck_kernel<K, FSM_VAR, false>;
+}
+
+KernelFn FSM_CAT(get_kernel_, FSM_VAR_NAME)(int K, bool split)
 {
     switch (K) {
-    case 1: return speck_kernel<1, FSM_VAR>;
-    case 2: return speck_kernel<2, FSM_VAR>;
-    case 3: return speck_kernel<3, FSM_VAR>;
-    case 4: return speck_kernel<4, FSM_VAR>;
-    case 6: return speck_kernel<6, FSM_VAR>;
-    case 8: return speck_kernel<8, FSM_VAR>;
-    case 12: return speck_kernel<12, FSM_VAR>;
-    default: return speck_kernel<16, FSM_VAR>;
+    case 1: return pick<1>(split);
+    case 2: return pick<2>(split);
+    case 3: return pick<3>(split);
+    case 4: return pick<4>(split);
+    case 6: return pick<6>(split);
+    case 8: return pick<8>(split);
+    case 12: return pick<12>(split);
+    default: return pick<16>(split);
     }
 }
 

@@ -825,7 +825,9 @@ __device__ __forceinline__ void named_arrive(uint32_t id, uint32_t n)
 // (HTML, k = 1: +13 %, its serial re-executions dominate the epilogue) and the multi-chain kernels
 // of the shared-memory variants (P4 / P8 / B, K >= 2: +6..15 %).  K = 1 kernels of P8 / B / G / HS
 // lose more from the missing 32nd worker warp and stash than they gain (-4..-8 %): unsplit.
-// FSM_SPLIT: 2 = this policy (default), 1 = always, 0 = never (experiments).
+// FSM_SPLIT: 2 = this policy (default), 1 = always, 0 = never (experiments).  A launch runs split
+// only if the policy says so AND the double-buffered layout fits in shared memory (large-K CL
+// kernels next to a 150 KiB table do not).
 #ifndef FSM_SPLIT
 #define FSM_SPLIT 2
 #endif
@@ -1478,10 +1480,11 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
     }
 }
 
-template <int K, int VAR>
+// SPLIT is chosen per launch by the host: split_kernel(VAR, K) and the double-buffered layout fits.
+template <int K, int VAR, bool SPLIT>
 __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Params p)
 {
-    speck_body<K, VAR, false, split_kernel(VAR, K)>(p, nullptr, 1);
+    speck_body<K, VAR, false, SPLIT>(p, nullptr, 1);
 }
 
 template <int K, int VAR>

@@ -428,3 +428,15 @@ def test_run_multi_matches_single_runs():
         for f in fs:
             f.close()
         torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("k", [6, 8, 12, 16])
+def test_html_cl_large_k(k):
+    """Large-K CL kernels: the split (epilogue-warp) layout does not fit next to the 146 KiB class
+    table for every K, so those launches fall back to the unsplit kernel; both are exact."""
+    d = dfas.html_tokenizer()
+    data = streams.html_bytes(3_000_001, 71 + k)
+    exp = seq.run(d, data)
+    for lb in (0, 64):
+        got, st = gpu_run(d, data, k=k, variant=VARIANTS["CL"], lookback_len=lb)
+        assert got == exp, (k, lb, st)

@@ -379,6 +379,28 @@ def main():
     }
     if tuning is not None:
         line["tuning"] = {kk: (round(v, 3) if isinstance(v, float) else v) for kk, v in tuning.items()}
+    # achievable HBM read ceiling on the same buffer (read-only streaming kernel)
+    if world == 1 and n >= (1 << 30):
+        from fsmgen import _native
+        sink = torch.zeros(4, dtype=torch.int32, device=dev)
+        rs = []
+        for i in range(4):
+            if flush is not None:
+                flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            rc = _native.dev_lib().fsmgen_dev_read_stream(buf.data_ptr(), n, sink.data_ptr(),
+                                                          torch.cuda.get_device_properties(dev).multi_processor_count,
+                                                          stream.cuda_stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            if rc == 0 and i:
+                rs.append(e0.elapsed_time(e1) / 1e3)
+        if rs:
+            rgbs = (n // 32 * 32) / statistics.median(rs) / 1e9
+            line["roofline"]["read_ceiling"] = {"value": round(rgbs, 1), "unit": "GB/s",
+                                                "frac": round((n / step_s / 1e9) / rgbs, 4),
+                                                "kernel": "read-only LDG.256 stream over the same input"}
     if not args.no_ablation and world == 1:
         # internal ablation: the paper's sequential merge (Fig. 4a) on the same input and chains
         f.set_options(variant=args.variant, chunk_bytes=args.chunk, merge=fsmspec.FSM_MERGE_SEQUENTIAL,

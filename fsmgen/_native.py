@@ -67,5 +67,8 @@ def dev_lib() -> ctypes.CDLL:
         lib.fsmgen_dev_fill.restype = ctypes.c_int
         lib.fsmgen_dev_fill.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64,
                                         ctypes.c_uint64, ctypes.c_void_p]
+        lib.fsmgen_dev_read_stream.restype = ctypes.c_int
+        lib.fsmgen_dev_read_stream.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_int,
+                                               ctypes.c_void_p]
         _dev = lib
     return _dev

@@ -32,7 +32,44 @@ __global__ void fill_bytes(uint8_t *__restrict__ out, uint64_t seed, uint64_t of
         out[i] = (uint8_t)(mix64(seed + ((j >> 3) + 1) * kGolden) >> (8 * (j & 7)));
     }
 }
+// Measurement helper: a read-only streaming kernel over the same input -- 32-byte
+// non-coherent loads, 4 in flight per thread, XOR-folded into one word per thread so nothing is
+// elided.  Its GB/s is the achievable HBM *read* ceiling the FSM kernel is compared against (the
+// MEASURED_PEAKS figure is a copy, read + write).
+__global__ void read_stream(const uint8_t *__restrict__ in, uint64_t n32, uint32_t *__restrict__ sink)
+{
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t acc = 0;
+    for (; i + 3 * stride < n32; i += 4 * stride) {
+        uint32_t v[4][8];
+#pragma unroll
+        for (int u = 0; u < 4; u++)
+            asm volatile("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                         : "=r"(v[u][0]), "=r"(v[u][1]), "=r"(v[u][2]), "=r"(v[u][3]), "=r"(v[u][4]),
+                           "=r"(v[u][5]), "=r"(v[u][6]), "=r"(v[u][7])
+                         : "l"(in + 32 * (i + u * stride)));
+#pragma unroll
+        for (int u = 0; u < 4; u++)
+#pragma unroll
+            for (int w = 0; w < 8; w++) acc ^= v[u][w];
+    }
+    for (; i < n32; i += stride) {
+        const uint4 *q = reinterpret_cast<const uint4 *>(in + 32 * i);
+        const uint4 a = __ldg(q), b = __ldg(q + 1);
+        acc ^= a.x ^ a.y ^ a.z ^ a.w ^ b.x ^ b.y ^ b.z ^ b.w;
+    }
+    if (acc == 0x9E3779B9u) sink[0] = acc;  // practically never taken; keeps the loads live
+}
 } // namespace
+
+// Read-only streaming pass over n bytes (32-byte aligned pointer, n multiple of 32 used).
+extern "C" int fsmgen_dev_read_stream(const void *dev_in, uint64_t n, void *dev_sink, int num_sms, void *stream)
+{
+    const uint64_t n32 = n / 32;
+    read_stream<<<num_sms * 8, 256, 0, (cudaStream_t)stream>>>((const uint8_t *)dev_in, n32, (uint32_t *)dev_sink);
+    return cudaGetLastError() == cudaSuccess ? 0 : -3;
+}
 
 extern "C" int fsmgen_dev_fill(void *dev_out, uint64_t seed, uint64_t offset, uint64_t len, void *stream)
 {

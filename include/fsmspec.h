@@ -56,8 +56,10 @@ enum {
     FSM_VARIANT_H8 = 4,  /* N <= 8 (byte mode): half rows of 4 states, one LDS.32 per chain step   */
     FSM_VARIANT_HS = 5,  /* byte mode, N <= 32768: hot-state row caching (Sec. 4.2): the most frequent
                             states' rows in shared memory (u16), the rest from the u32 table in L2 */
-    FSM_VARIANT_CL = 6   /* N x byte-classes <= 1024: class-compressed, lane-replicated table, one
+    FSM_VARIANT_CL = 6,  /* N x byte-classes <= 1024: class-compressed, lane-replicated table, one
                             conflict-free LDS.32 per chain step (e.g. the HTML tokenizer) */
+    FSM_VARIANT_N8 = 7   /* N <= 8 (byte mode): one u32 row of eight 4-bit fields per symbol, lane-replicated
+                            smem (one LDS.32 per byte), chain = wrap-mode funnel shift + IMAD          */
 };
 
 /* Merge strategies: the paper's parallel merge (default) and its sequential-merge baseline

@@ -51,6 +51,7 @@ FSM_DECLARE_VARIANT(b)
 FSM_DECLARE_VARIANT(g)
 FSM_DECLARE_VARIANT(hs)
 FSM_DECLARE_VARIANT(cl)
+FSM_DECLARE_VARIANT(n8)
 
 static KernelFn get_kernel(int var, int K, bool split)
 {
@@ -60,6 +61,7 @@ static KernelFn get_kernel(int var, int K, bool split)
     case VAR_H8: return get_kernel_h8(K, split);
     case VAR_HS: return get_kernel_hs(K, split);
     case VAR_CL: return get_kernel_cl(K, split);
+    case VAR_N8: return get_kernel_n8(K, split);
     case VAR_B: return get_kernel_b(K, split);
     default: return get_kernel_g(K, split);
     }
@@ -72,6 +74,7 @@ static MultiFn get_multi(int var, int K)
     case VAR_H8: return get_multi_h8(K);
     case VAR_HS: return get_multi_hs(K);
     case VAR_CL: return get_multi_cl(K);
+    case VAR_N8: return get_multi_n8(K);
     case VAR_B: return get_multi_b(K);
     default: return get_multi_g(K);
     }
@@ -84,6 +87,7 @@ static FixFn get_fix(int var)
     case VAR_H8: return get_fix_h8();
     case VAR_HS: return get_fix_hs();
     case VAR_CL: return get_fix_cl();
+    case VAR_N8: return get_fix_n8();
     case VAR_B: return get_fix_b();
     default: return get_fix_g();
     }
@@ -96,6 +100,7 @@ static SpecFn get_spec(int var)
     case VAR_H8: return get_spec_h8();
     case VAR_HS: return get_spec_hs();
     case VAR_CL: return get_spec_cl();
+    case VAR_N8: return get_spec_n8();
     case VAR_B: return get_spec_b();
     default: return get_spec_g();
     }
@@ -108,6 +113,7 @@ static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
     case VAR_H8: get_seq_h8(K, l, w); break;
     case VAR_HS: get_seq_hs(K, l, w); break;
     case VAR_CL: get_seq_cl(K, l, w); break;
+    case VAR_N8: get_seq_n8(K, l, w); break;
     case VAR_B: get_seq_b(K, l, w); break;
     default: get_seq_g(K, l, w); break;
     }
@@ -131,8 +137,8 @@ struct fsm {
     int auto_variant = VAR_G;
     fsm_options opt{};
     // device tables
-    void *d_img[7] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
-    uint32_t img_bytes[7] = {0, 0, 0, 0, 0, 0, 0};
+    void *d_img[8] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    uint32_t img_bytes[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     uint32_t ncls = 0, cl_magic = 0;  // CL variant
     // static-frequency renumbering (hot-state caching): user <-> internal ids
     bool renumbered = false;
@@ -225,7 +231,7 @@ extern "C" int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint
 
 static void free_all(fsm *f)
 {
-    for (int i = 0; i < 7; i++) cudaFree(f->d_img[i]);
+    for (int i = 0; i < 8; i++) cudaFree(f->d_img[i]);
     cudaFree(f->d_inv);
     cudaFree(f->d_lb);
     cudaFree(f->d_nimg);
@@ -327,6 +333,11 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         if ((rc = upload(&f->d_img[VAR_H8], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_H8] = 0;
     }
+    if (n <= 8 && !bits) {  // N8's count bit is byte-mode only
+        auto img = image_n8(f->dfa);
+        if ((rc = upload(&f->d_img[VAR_N8], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_N8] = 0;
+    }
     if (n <= 8) {
         auto img = image_packed(f->dfa, true);
         if ((rc = upload(&f->d_img[VAR_P8], img.data(), img.size()))) return fail(rc);
@@ -411,7 +422,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
-    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_CL) return FSM_EINVAL;
+    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_N8) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
@@ -570,6 +581,8 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     p.k_512 = 512;
     p.k_1e27 = 1u << 27;
     p.k_2 = 2;
+    p.k_4 = 4;
+    p.k_1e28 = 1u << 28;
     p.table_g = static_cast<const uint32_t *>(f->d_img[VAR_G]);
     p.hot_rows = f->hot_rows;
     p.inv = f->d_inv;
@@ -885,7 +898,7 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
     }
     fp.out = f->d_fix;
     fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows,
-                   f->ncls, f->cl_magic};
+                   f->ncls, f->cl_magic, 4, 1u << 28};
     FixFn fn = get_fix(var);
     const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

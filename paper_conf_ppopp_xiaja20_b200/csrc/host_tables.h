@@ -197,6 +197,19 @@ inline std::vector<uint8_t> image_h8(const ByteDFA &d)
     return img;
 }
 
+// N8 (byte mode, N <= 8): per symbol one u32 row of 4-bit fields, field s = next | count << 3.
+inline std::vector<uint8_t> image_n8(const ByteDFA &d)
+{
+    std::vector<uint8_t> img(256 * 4, 0);
+    uint32_t *p = reinterpret_cast<uint32_t *>(img.data());
+    for (uint32_t c = 0; c < 256; c++)
+        for (uint32_t s = 0; s < d.n; s++) {
+            const uint32_t nx = d.next[(size_t)s * 256 + c], k = d.inc[(size_t)s * 256 + c];
+            p[c] |= (nx | (k << 3)) << (4 * s);
+        }
+    return img;
+}
+
 inline std::vector<uint8_t> image_b(const ByteDFA &d)
 {
     std::vector<uint8_t> img((size_t)d.n * 512);

@@ -27,7 +27,7 @@
 
 namespace speck {
 
-enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5, VAR_CL = 6 };
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5, VAR_CL = 6, VAR_N8 = 7 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
 // in lockstep over the chunk's first kExtWindow bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
@@ -154,7 +154,7 @@ __device__ __forceinline__ uint32_t dp4a_u(uint32_t a, uint32_t b, uint32_t c)
 }
 constexpr uint32_t kPackedBase = 0x10000u;  // shared-window address of the packed tables
 constexpr uint32_t kSmemWindowBase = 1024u;  // dynamic shared memory starts here (measured: tools/smem_probe)
-__host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1 || var == 4; }
+__host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1 || var == 4 || var == 7; }
 // Offset (from the start of dynamic smem) of the scratch area that follows the table.  Packed
 // tables occupy the window [0x10000, 0x20000); everything else goes above them.
 __host__ __device__ constexpr uint32_t scratch_offset(int var, uint32_t table_bytes)
@@ -176,10 +176,11 @@ struct KConst {
     const uint32_t *gtab;  // full u32 table in global memory (HS variant)
     uint32_t hot_rows;     // HS: states [0, hot_rows) have their rows in shared memory
     uint32_t ncls, cl_magic;  // CL: byte classes, ceil(2^32 / ncls)
+    uint32_t k_4, k_1e28;     // N8
 };
 __device__ __forceinline__ KConst kconst(const Params &p)
 {
-    return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2, p.table_g, p.hot_rows, p.ncls, p.cl_magic};
+    return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2, p.table_g, p.hot_rows, p.ncls, p.cl_magic, p.k_4, p.k_1e28};
 }
 
 // ------------------------------------------------------------------- table-placement variants --
@@ -320,6 +321,65 @@ struct TableH8 {
         const uint32_t f = prmt(w, w, st & 3u) & 0xFFu;
         cnt += (f >> 4) & 1u;
         return (f & 3u) | ((f >> 5) & 4u);
+    }
+};
+
+// N8: N <= 8, byte mode.  The transition function of symbol c is ONE 32-bit row of eight 4-bit
+// fields, field s = next | count << 3, lane-replicated at 0x10000 + c * 256 + lane * 4 (P4's layout,
+// so the address is one PRMT of the input word and the load is one conflict-free LDS.32 = one
+// wavefront per byte per warp, half of P8's LDS.64).  A chain carries the shift amount 4 * state:
+// t = funnel-shift-right(row, cur) in wrap mode (only cur & 31 is used), and the next shift amount
+// is t * 4, whose bits 2..4 are t's next-state bits -- the garbage above bit 4 is ignored by the
+// next wrap-mode shift.  Chain step: SHF.R.W (ALU) + IMAD (FMA); count bit = bit 3 of t, added on
+// the ALU (LOP3 + half an IADD3) and FMA (IMAD + IMAD.HI) pipes on alternate steps.
+struct TableN8 {
+    uint32_t lanereg;
+    uint32_t c4, c28, c2;
+    __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
+    {
+        lanereg = kPackedBase | ((threadIdx.x & 31) * 4);
+        c4 = kc.k_4;
+        c28 = kc.k_1e28;
+        c2 = kc.k_2;
+        const uint32_t *rows = static_cast<const uint32_t *>(g);
+        for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
+            const uint32_t v = __ldg(rows + (i >> 5));
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(kPackedBase + (i >> 5) * 256 + (i & 31) * 4), "r"(v));
+        }
+    }
+    __device__ __forceinline__ static uint32_t shr_wrap(uint32_t row, uint32_t sh)
+    {
+        uint32_t d;
+        asm("shf.r.wrap.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(row), "r"(0u), "r"(sh));
+        return d;
+    }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st * 4u; }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return (cur >> 2) & 7u; }
+    // acc = 8 * (ALU-counted steps), accf = FMA-counted steps
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const
+    {
+        return (acc >> 3) + accf;
+    }
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
+    {
+        const uint32_t r = lds_u32(prmt(w, lanereg, 0x7604u | (uint32_t(j) << 4)));
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            const uint32_t t = shr_wrap(r, cur[s]);          // field of the current state in bits 0..3
+            cur[s] = mad_lo(t, c4, 0u);                      // next shift amount (bits 2..4 valid)
+            if (((j + s) & 1) == 0) acc[s] += t & 8u;        // ALU: LOP3 (+ half an IADD3)
+            else accf[s] = mad_hi(t * c28, c2, accf[s]);     // FMA: IMAD, IMAD.HI (bit 3 of t)
+        }
+    }
+    using Row = uint32_t;
+    __device__ __forceinline__ Row row(uint32_t c) const { return lds_u32(lanereg + (c << 8)); }
+    __device__ __forceinline__ uint32_t apply(Row r, uint32_t st, uint32_t &cnt) const
+    {
+        const uint32_t f = (r >> (4 * st)) & 0xFu;
+        cnt += f >> 3;
+        return f & 7u;
     }
 };
 
@@ -503,6 +563,7 @@ template <> struct TableFor<VAR_G> { using type = TableG; };
 template <> struct TableFor<VAR_H8> { using type = TableH8; };
 template <> struct TableFor<VAR_HS> { using type = TableHS; };
 template <> struct TableFor<VAR_CL> { using type = TableCL; };
+template <> struct TableFor<VAR_N8> { using type = TableN8; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <int K, class TB>
@@ -835,7 +896,7 @@ __host__ __device__ constexpr bool split_kernel(int var, int K)
 {
     return FSM_SPLIT == 1 ? true
          : FSM_SPLIT == 0 ? false
-         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 4 || var == 2) /* P4 P8 H8 B */ && K >= 2));
+         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 4 || var == 2 || var == 7) /* P4 P8 H8 B N8 */ && K >= 2));
 }
 
 // Per-tile context used by re-execution and the epilogue.

@@ -89,6 +89,7 @@ struct Params {
     uint32_t ncls, cl_magic;       // CL variant: byte classes and ceil(2^32 / ncls)
     uint32_t *user_out;            // optional: the last tile also writes {user state, 0, count lo, hi} here
     uint32_t eager_window;         // NEXT-3 eager completion: bytes of lockstep per chunk (0 = off)
+    uint32_t k_4, k_1e28;          // N8 variant: FMA-pipe constants (4, 1 << 28), see k_1e24 above
 };
 
 }  // namespace speck

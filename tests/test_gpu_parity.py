@@ -35,12 +35,13 @@ def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
     return res, st
 
 
-VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4, "HS": 5, "CL": 6}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4, "HS": 5, "CL": 6, "N8": 7}
 
 
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
     return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "H8": n <= 8 and not dfa.bit_mode,
+            "N8": n <= 8 and not dfa.bit_mode,
             "B": n <= 256, "G": True, "HS": not dfa.bit_mode and n <= 32768,
             "CL": _n_classes(dfa) >= 2 and n * ((_n_classes(dfa) + 1) & ~1) <= 1024}[var]
 
@@ -69,7 +70,7 @@ def _n_classes(dfa):
 
 
 # --------------------------------------------------------------------- worked example on GPU
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS", "CL"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "N8", "B", "G", "HS", "CL"])
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
 def test_fig1_worked_example(var, k):
     d = dfas.c_comment(True)
@@ -79,7 +80,7 @@ def test_fig1_worked_example(var, k):
 
 
 # --------------------------------------------------------------------- C1-shaped text
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "B", "G", "HS", "CL"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "N8", "B", "G", "HS", "CL"])
 @pytest.mark.parametrize("chunk", [0, 64, 96, 4096])
 def test_c_comment_text(var, chunk):
     d = dfas.c_comment(True)

@@ -195,6 +195,53 @@ def config_json(args, w):
             "l2": "input >> L2 (126 MB), no flush needed" if w["total"] > 4 * 126e6 else "L2 flushed between steps"}
 
 
+def certify_full(args, w, f, buf, n, k, final):
+    """Full-length parity of the timed configuration, part of the CPU-baseline leg.
+    The GPU claims the state at G segment boundaries (chained fsm_run_shard maps + fixups); every
+    host core runs the plain sequential loop (oracle) over its segment from the claimed start,
+    streaming the regenerated input; the check passes iff segment 0 starts in q0, each segment
+    ends where the next one claims to start, and the chained (end, count) equals the fused
+    kernel's result.  By induction that is the sequential oracle over the whole input."""
+    import concurrent.futures as cf
+
+    from fsmgen import streams
+    from oracle import seq
+
+    t0 = time.perf_counter()
+    d = w["dfa"]
+    G = max(1, min(os.cpu_count() or 1, 32))
+    bounds = [n * g // G // 32 * 32 for g in range(G)] + [n]
+    claims, x = [], d.start
+    for g in range(G):
+        lo, hi = bounds[g], bounds[g + 1]
+        claims.append(x)
+        m, sh = f.run_shard(buf.data_ptr() + lo, hi - lo, halo=(buf.data_ptr() + lo - 1) if g else None,
+                            halo_len=1 if g else 0, k=k, keep=True)
+        hit = [(e, c) for s, e, c in m.slots() if s == x]
+        x = hit[0][0] if hit else f.shard_fixup(sh, x)[0]
+        sh.close()
+    sseed = streams.MASTER_SEED + 5
+    piece = 1 << 28
+
+    def segment(g):
+        lo, hi = bounds[g], bounds[g + 1]
+        st, total = claims[g], 0
+        tmp = np.empty(piece, dtype=np.uint8)
+        for o in range(lo, hi, piece):
+            m_ = min(piece, hi - o)
+            st, c = seq.run_from(d, st, streams.splitmix_bytes(sseed, o, m_, out=tmp), m_)
+            total += c
+        return st, total
+
+    with cf.ThreadPoolExecutor(G) as ex:
+        res = list(ex.map(segment, range(G)))
+    ok = claims[0] == d.start and all(res[g][0] == claims[g + 1] for g in range(G - 1))
+    end, total = res[-1][0], sum(c for _, c in res)
+    ok = ok and (end, total) == tuple(final)
+    return {"bytes": n, "segments": G, "cores": G, "ok": bool(ok), "seconds": round(time.perf_counter() - t0, 1),
+            "method": "GPU-claimed segment starts, oracle loop per segment on its own core (induction)"}
+
+
 # ----------------------------------------------------------------------------- our arm
 def main():
     ap = argparse.ArgumentParser()
@@ -211,6 +258,7 @@ def main():
     ap.add_argument("--size-gib", type=float, default=0.0, help="input size (default: the config's)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-certify", action="store_true", help="skip the full-length certificate (C5)")
     ap.add_argument("--variant", type=int, default=-1)
     ap.add_argument("--lookback", type=int, default=-1,
                     help="look-back window bytes (R7; -1 = the config's default: c5 0, c1/c4 64, c2/c3 32)")
@@ -372,7 +420,9 @@ def main():
                      "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback"},
         "traffic_note": "ncu --set full (profiles/r01_ncu_c5_n8m2k2_8GiB.txt): dram read+write = 1.037 x input bytes (8.881 GB read + 0.030 GB written for 8 GiB)",
         "clocks": clk.summary(),
-        "gpu_launches": args.steps,  # one fused kernel per step (plus a fix-up kernel per miss round for N > 1)
+        # one fused kernel per step, plus the look-back window pre-pass when the window is >= 32 bytes
+        # (and, for N > 1, a fix-up kernel per shard-boundary miss round)
+        "gpu_launches": args.steps * (2 if (lookback or 0) >= 32 else 1),
         "result": {"final_state": final[0], "accept_count": final[1]},
         "stats": {kk: v for kk, v in st.items()},
         "e2e": e2e,
@@ -432,6 +482,8 @@ def main():
                                 "sample": f"first {cb['bytes']} bytes of the workload ({cb['seconds']:.1f} s)"}
         line["parity_sample"] = {"bytes": cb["bytes"], "ok": gp == cb["result"]}
         line["host_cores"] = os.cpu_count()
+        if "host" in w and not args.no_certify:
+            line["parity_full"] = certify_full(args, w, f, buf, n, k, final)
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

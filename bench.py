@@ -106,23 +106,34 @@ class ClockSampler:
 
     def __init__(self, index: int):
         self.index = index
-        self.rows = []
+        self.rows = []      # (arrival time, fields)
         self.proc = None
+        self.window = None  # (start, end) of the timed region, time.monotonic()
 
     def __enter__(self):
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "20"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            t0 = time.monotonic()
+            while not self.rows and time.monotonic() - t0 < 5.0:  # sampler running before timing starts
+                time.sleep(0.01)
         except OSError:
             self.proc = None
         return self
 
     def _read(self):
         for line in self.proc.stdout:
-            self.rows.append([x.strip() for x in line.split(",")])
+            self.rows.append((time.monotonic(), [x.strip() for x in line.split(",")]))
+
+    def start(self):
+        self.window = [time.monotonic(), None]
+
+    def stop(self):
+        time.sleep(0.05)  # let the sample covering the end arrive
+        self.window[1] = time.monotonic()
 
     def __exit__(self, *a):
         if self.proc:
@@ -130,11 +141,17 @@ class ClockSampler:
             self.proc.wait()
 
     def summary(self):
-        sm = [float(r[0]) for r in self.rows if r and r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
+        rows = self.rows
+        if self.window and self.window[1]:
+            inside = [r for t, r in rows if self.window[0] <= t <= self.window[1]]
+            rows = inside if inside else [r for _, r in rows[-2:]]
+        else:
+            rows = [r for _, r in rows]
+        sm = [float(r[0]) for r in rows if r and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
         reasons = set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in self.rows:
+        for r in rows:
             for i, nme in enumerate(names):
                 if len(r) > 4 + i and r[4 + i].lower() == "active":
                     reasons.add(nme)
@@ -341,6 +358,7 @@ def main():
         dist.barrier()
     times = []
     with ClockSampler(local) as clk:
+        clk.start()
         for _ in range(args.steps):
             if flush is not None:
                 flush.zero_()
@@ -354,6 +372,7 @@ def main():
             e1.record(stream)
             torch.cuda.synchronize()
             times.append(e0.elapsed_time(e1) / 1e3)
+        clk.stop()
     t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -472,10 +491,13 @@ def main():
                             "paper_v100_context": "2.02-6.74x (P:11, P:53)"}
     if not args.no_cpu and world == 1:
         try:
-            os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+            all_cores = os.sched_getaffinity(0)
+            os.sched_setaffinity(0, {sorted(all_cores)[0]})  # the 1-core oracle baseline
         except (AttributeError, OSError):
-            pass
+            all_cores = None
         cb = cpu_oracle_rate(w, budget_s=12.0)
+        if all_cores:
+            os.sched_setaffinity(0, all_cores)  # the certificate below uses every core
         # parity on the sampled prefix: the GPU runs the same prefix in the bench's configuration
         gp = f.run_spec_k(buf.data_ptr(), cb["bytes"] * (8 if w["bits"] else 1), k)
         line["cpu_baseline"] = {"value": round(cb["gbs"], 4), "unit": "GB/s", "cores": 1, "kind": "oracle",

@@ -308,7 +308,10 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
     // N > 256: the u32 table in L2 with the L1 acting as a hardware hot-row cache (G) measured faster
     // up to ~2K states (1027-state AC: 1.12 vs 0.98 TB/s); beyond that explicit hot-state caching in
     // shared memory wins (4121-state AC: 0.90 vs 0.76 TB/s).  Both use the frequency renumbering.
-    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B
+    // N <= 8 in byte mode: N8 (4-bit fields, one LDS.32 per byte, batched DP4A counts) measured
+    // +15..28 % over P8 (LDS.64-bound) on (8, m, k) DFAs; P4 stays ahead for N <= 4; bit mode has
+    // up to 8 accepts per byte, which N8's 1-bit count field cannot hold, so it keeps P8.
+    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : (n <= 8 && !bits) ? VAR_N8 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B
                     : (f->renumbered && n > 2048) ? VAR_HS : VAR_G;
     f->opt.chunk_bytes = 0;
     f->opt.threads_per_tile = 0;  // auto: max_threads(K)

@@ -355,10 +355,12 @@ struct TableN8 {
     }
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st * 4u; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return (cur >> 2) & 7u; }
-    // acc = 8 * (ALU-counted steps), accf = FMA-counted steps
+    // acc = 8 * (ALU-counted steps) + 32 * (step4-counted steps): the two never mix in one chunk's
+    // 32-byte blocks (step4) and its byte tail (step), and 8 | 32, so acc / 8 ... is exact only if
+    // the batched part is kept apart -- it is: step4 adds into accf (units of 32), step into acc.
     __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const
     {
-        return (acc >> 3) + accf;
+        return (acc >> 3) + (kStep4 ? (accf >> 5) : accf);
     }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
@@ -369,8 +371,36 @@ struct TableN8 {
         for (int s = 0; s < K; s++) {
             const uint32_t t = shr_wrap(r, cur[s]);          // field of the current state in bits 0..3
             cur[s] = mad_lo(t, c4, 0u);                      // next shift amount (bits 2..4 valid)
-            if (((j + s) & 1) == 0) acc[s] += t & 8u;        // ALU: LOP3 (+ half an IADD3)
-            else accf[s] = mad_hi(t * c28, c2, accf[s]);     // FMA: IMAD, IMAD.HI (bit 3 of t)
+            if (kStep4 || ((j + s) & 1) == 0) acc[s] += t & 8u;  // ALU: LOP3 (+ half an IADD3)
+            else accf[s] = mad_hi(t * c28, c2, accf[s]);          // FMA: IMAD, IMAD.HI (bit 3 of t)
+        }
+    }
+#ifndef FSM_N8_BATCH
+#define FSM_N8_BATCH 1
+#endif
+    // Four bytes of word w at once: the four rows are loaded up front, and the count of the four
+    // steps is taken in one go -- the next shift amounts v = 4t carry the accept bit in bit 5; their
+    // low bytes are gathered by two PRMTs into one word, masked, and summed by one DP4A (acc counts
+    // in units of 32).  ALU: 4 address PRMT + 4 SHF + 3 PRMT + 1 LOP3; FMA: 4 IMAD + 1 DP4A.
+    static constexpr bool kStep4 = FSM_N8_BATCH != 0;
+    template <int K>
+    __device__ __forceinline__ void step4(uint32_t w, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    {
+        uint32_t r[4];
+#pragma unroll
+        for (int j = 0; j < 4; j++) r[j] = lds_u32(prmt(w, lanereg, 0x7604u | (uint32_t(j) << 4)));
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            uint32_t v[4];
+            uint32_t c = cur[s];
+#pragma unroll
+            for (int j = 0; j < 4; j++) {
+                v[j] = mad_lo(shr_wrap(r[j], c), c4, 0u);
+                c = v[j];
+            }
+            cur[s] = c;
+            const uint32_t lo = prmt(v[0], v[1], 0x0040u), hi = prmt(v[2], v[3], 0x0040u);
+            acc[s] = dp4a_u(prmt(lo, hi, 0x5410u) & 0x20202020u, 0x01010101u, acc[s]);
         }
     }
     using Row = uint32_t;
@@ -566,11 +596,17 @@ template <> struct TableFor<VAR_CL> { using type = TableCL; };
 template <> struct TableFor<VAR_N8> { using type = TableN8; };
 
 // --------------------------------------------------------------------- a4: local processing --
+template <class TB> struct TableHasStep4 { static constexpr bool value = false; };
+template <> struct TableHasStep4<TableN8> { static constexpr bool value = TableN8::kStep4; };
+
 template <int K, class TB>
 __device__ __forceinline__ void process32(const TB &tb, const Bytes32 &x, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                           uint32_t (&accf)[K])
 {
-    if constexpr (K <= 4) {
+    if constexpr (TableHasStep4<TB>::value) {
+#pragma unroll
+        for (int q = 0; q < 8; q++) tb.template step4<K>(x.w[q], cur, accf);
+    } else if constexpr (K <= 4) {
 #pragma unroll
         for (int q = 0; q < 8; q++)
 #pragma unroll

@@ -334,13 +334,17 @@ struct TableH8 {
 // the ALU (LOP3 + half an IADD3) and FMA (IMAD + IMAD.HI) pipes on alternate steps.
 struct TableN8 {
     uint32_t lanereg;
-    uint32_t c4, c28, c2;
+    uint32_t c4, c28, c2, c24, c16x, c8x, c256;
     __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
     {
         lanereg = kPackedBase | ((threadIdx.x & 31) * 4);
         c4 = kc.k_4;
         c28 = kc.k_1e28;
         c2 = kc.k_2;
+        c24 = kc.k_1e24;          // 1 << 24
+        c16x = kc.k_16 << 12;     // 1 << 16
+        c8x = kc.k_16 << 4;       // 1 << 8
+        c256 = kc.k_512 >> 1;     // 256
         const uint32_t *rows = static_cast<const uint32_t *>(g);
         for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
             const uint32_t v = __ldg(rows + (i >> 5));
@@ -378,6 +382,9 @@ struct TableN8 {
 #ifndef FSM_N8_BATCH
 #define FSM_N8_BATCH 1
 #endif
+#ifndef FSM_N8_FMA_ADDR
+#define FSM_N8_FMA_ADDR 0
+#endif
     // Four bytes of word w at once: the four rows are loaded up front, and the count of the four
     // steps is taken in one go -- the next shift amounts v = 4t carry the accept bit in bit 5; their
     // low bytes are gathered by two PRMTs into one word, masked, and summed by one DP4A (acc counts
@@ -387,8 +394,17 @@ struct TableN8 {
     __device__ __forceinline__ void step4(uint32_t w, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
     {
         uint32_t r[4];
+#if FSM_N8_FMA_ADDR
+        // bytes 0 and 3 addressed on the FMA pipe (the ALU pipe is the binding one):
+        //   byte 0: x = w << 24 (IMAD), addr = (x >> 16) + lanereg (IMAD.HI);  byte 3: (w >> 24) * 256 + lanereg
+        r[0] = lds_u32(mad_hi(mad_lo(w, c24, 0u), c16x, lanereg));
+        r[1] = lds_u32(prmt(w, lanereg, 0x7614u));
+        r[2] = lds_u32(prmt(w, lanereg, 0x7624u));
+        r[3] = lds_u32(mad_lo(mad_hi(w, c8x, 0u), c256, lanereg));
+#else
 #pragma unroll
         for (int j = 0; j < 4; j++) r[j] = lds_u32(prmt(w, lanereg, 0x7604u | (uint32_t(j) << 4)));
+#endif
 #pragma unroll
         for (int s = 0; s < K; s++) {
             uint32_t v[4];

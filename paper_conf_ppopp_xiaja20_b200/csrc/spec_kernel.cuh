@@ -36,25 +36,33 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
         } else if (b >= Lw + 1 && p.aligned) {
             const uint32_t c0 = __ldg(p.in + b - Lw - 1);
             const uint32_t ni = __ldg(p.nimg + c0);
-            uint32_t y[KMAX];
+            // the image chains run in the table variant's own hot-loop form (its step(), on groups of
+            // 4 chains, only as many groups as the image has states); ids are recovered at the end
+            uint32_t cur[KMAX / 4][4], acc[KMAX / 4][4], accf[KMAX / 4][4];
 #pragma unroll
-            for (int i = 0; i < KMAX; i++) y[i] = (uint32_t)__ldg(p.lb + c0 * KMAX + ((uint32_t)i < ni ? i : 0));
+            for (int q0 = 0; q0 < KMAX / 4; q0++)
+#pragma unroll
+                for (int i = 0; i < 4; i++) {
+                    const int ii = q0 * 4 + i;
+                    cur[q0][i] = tb.init((uint32_t)__ldg(p.lb + c0 * KMAX + ((uint32_t)ii < ni ? ii : 0)));
+                    acc[q0][i] = accf[q0][i] = 0;
+                }
             for (uint32_t o = 0; o < Lw; o += 32) {
                 const Bytes32 x = ldg256(p.in + b - Lw + o);
-#pragma unroll 1
-                for (int t = 0; t < 32; t++) {
-                    const uint32_t byte = (x.w[t >> 2] >> (8 * (t & 3))) & 0xFFu;
-                    const typename TB::Row r = tb.row(byte);
-                    uint32_t dummy = 0;
-                    // only the image's ni chains are live: skip whole groups of 4 beyond it
 #pragma unroll
-                    for (int q0 = 0; q0 < KMAX; q0 += 4)
-                        if ((uint32_t)q0 < ni) {
+                for (int q = 0; q < 8; q++) {
 #pragma unroll
-                            for (int i = q0; i < q0 + 4; i++) y[i] = tb.apply(r, y[i], dummy);
-                        }
+                    for (int j = 0; j < 4; j++)
+#pragma unroll
+                        for (int q0 = 0; q0 < KMAX / 4; q0++)
+                            if ((uint32_t)(q0 * 4) < ni) tb.template step<4>(x.w[q], j, cur[q0], acc[q0], accf[q0]);
                 }
             }
+            uint32_t y[KMAX];
+#pragma unroll
+            for (int q0 = 0; q0 < KMAX / 4; q0++)
+#pragma unroll
+                for (int i = 0; i < 4; i++) y[q0 * 4 + i] = tb.state_of(cur[q0][i]);
             uint32_t mult[KMAX];
 #pragma unroll
             for (int i = 0; i < KMAX; i++) {

@@ -334,7 +334,7 @@ struct TableH8 {
 // the ALU (LOP3 + half an IADD3) and FMA (IMAD + IMAD.HI) pipes on alternate steps.
 struct TableN8 {
     uint32_t lanereg;
-    uint32_t c4, c28, c2, c24, c16x, c8x, c256;
+    uint32_t c4, c28, c2, c24, c16x, c8x, c256, c26;
     __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
     {
         lanereg = kPackedBase | ((threadIdx.x & 31) * 4);
@@ -345,6 +345,7 @@ struct TableN8 {
         c16x = kc.k_16 << 12;     // 1 << 16
         c8x = kc.k_16 << 4;       // 1 << 8
         c256 = kc.k_512 >> 1;     // 256
+        c26 = kc.k_1e24 << 2;     // 1 << 26
         const uint32_t *rows = static_cast<const uint32_t *>(g);
         for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
             const uint32_t v = __ldg(rows + (i >> 5));
@@ -359,12 +360,12 @@ struct TableN8 {
     }
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st * 4u; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return (cur >> 2) & 7u; }
-    // acc = 8 * (ALU-counted steps) + 32 * (step4-counted steps): the two never mix in one chunk's
-    // 32-byte blocks (step4) and its byte tail (step), and 8 | 32, so acc / 8 ... is exact only if
-    // the batched part is kept apart -- it is: step4 adds into accf (units of 32), step into acc.
+    // Without step4: acc = 8 * (ALU-counted steps), accf = FMA-counted steps.  With step4: accf
+    // counts in units of 32 (DP4A / LOP3 of bit 5 of v, and the byte tail), acc in units of 1 (the
+    // hybrid FSM_N8_BATCH == 2 FMA part).
     __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const
     {
-        return (acc >> 3) + (kStep4 ? (accf >> 5) : accf);
+        return kStep4 ? acc + (accf >> 5) : (acc >> 3) + accf;
     }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
@@ -375,7 +376,8 @@ struct TableN8 {
         for (int s = 0; s < K; s++) {
             const uint32_t t = shr_wrap(r, cur[s]);          // field of the current state in bits 0..3
             cur[s] = mad_lo(t, c4, 0u);                      // next shift amount (bits 2..4 valid)
-            if (kStep4 || ((j + s) & 1) == 0) acc[s] += t & 8u;  // ALU: LOP3 (+ half an IADD3)
+            if (kStep4) accf[s] += (t & 8u) << 2;                 // byte tails of step4 chunks: units of 32
+            else if (((j + s) & 1) == 0) acc[s] += t & 8u;        // ALU: LOP3 (+ half an IADD3)
             else accf[s] = mad_hi(t * c28, c2, accf[s]);          // FMA: IMAD, IMAD.HI (bit 3 of t)
         }
     }
@@ -391,7 +393,7 @@ struct TableN8 {
     // in units of 32).  ALU: 4 address PRMT + 4 SHF + 3 PRMT + 1 LOP3; FMA: 4 IMAD + 1 DP4A.
     static constexpr bool kStep4 = FSM_N8_BATCH != 0;
     template <int K>
-    __device__ __forceinline__ void step4(uint32_t w, uint32_t (&cur)[K], uint32_t (&acc)[K]) const
+    __device__ __forceinline__ void step4(uint32_t w, uint32_t (&cur)[K], uint32_t (&acc)[K], uint32_t (&accf2)[K]) const
     {
         uint32_t r[4];
 #if FSM_N8_FMA_ADDR
@@ -415,8 +417,16 @@ struct TableN8 {
                 c = v[j];
             }
             cur[s] = c;
+#if FSM_N8_BATCH == 2
+            // hybrid: steps 0, 1 counted on the FMA pipe (IMAD + IMAD.HI of bit 5 of v), steps 2, 3 on
+            // the ALU pipe (two LOP3 + one IADD3), in units of 32 -- moves work off the busy ALU pipe
+            accf2[s] = mad_hi(mad_lo(v[0], c26, 0u), c2, accf2[s]);
+            accf2[s] = mad_hi(mad_lo(v[1], c26, 0u), c2, accf2[s]);
+            acc[s] += (v[2] & 32u) + (v[3] & 32u);
+#else
             const uint32_t lo = prmt(v[0], v[1], 0x0040u), hi = prmt(v[2], v[3], 0x0040u);
             acc[s] = dp4a_u(prmt(lo, hi, 0x5410u) & 0x20202020u, 0x01010101u, acc[s]);
+#endif
         }
     }
     using Row = uint32_t;
@@ -621,7 +631,7 @@ __device__ __forceinline__ void process32(const TB &tb, const Bytes32 &x, uint32
 {
     if constexpr (TableHasStep4<TB>::value) {
 #pragma unroll
-        for (int q = 0; q < 8; q++) tb.template step4<K>(x.w[q], cur, accf);
+        for (int q = 0; q < 8; q++) tb.template step4<K>(x.w[q], cur, accf, acc);
     } else if constexpr (K <= 4) {
 #pragma unroll
         for (int q = 0; q < 8; q++)

@@ -367,10 +367,10 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         // CL: byte classes + lane-replicated class-compressed table when it fits shared memory
         std::vector<uint32_t> cls, rep;
         const uint32_t nc = cl_pad(byte_classes(f->dfa, cls, rep));
-        if (nc >= 2 && (uint64_t)f->dfa.n * nc <= 1024) {
+        if (nc >= 2 && (uint64_t)f->dfa.n * nc * 128 <= kClMaxTable) {  // entry table below the class map
             auto img = image_cl(f->dfa, cls, rep);
             if ((rc = upload(&f->d_img[VAR_CL], img.data(), img.size()))) return fail(rc);
-            f->img_bytes[VAR_CL] = (uint32_t)((256 + (size_t)f->dfa.n * nc) * 128);
+            f->img_bytes[VAR_CL] = (uint32_t)((size_t)f->dfa.n * nc * 128);
             f->ncls = nc;
             f->cl_magic = (uint32_t)((((uint64_t)1 << 32) + nc - 1) / nc);
             if (f->auto_variant == VAR_B) f->auto_variant = VAR_CL;

@@ -155,15 +155,23 @@ __device__ __forceinline__ uint32_t dp4a_u(uint32_t a, uint32_t b, uint32_t c)
 constexpr uint32_t kPackedBase = 0x10000u;  // shared-window address of the packed tables
 constexpr uint32_t kSmemWindowBase = 1024u;  // dynamic shared memory starts here (measured: tools/smem_probe)
 __host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1 || var == 4 || var == 7; }
+// CL: the entry table sits at the start of dynamic smem (shared address 0x400 up to < 0x20000) and
+// the 32 KiB lane-replicated class map at the fixed shared address 0x20000, so a class-map address
+// is (byte << 7) | lane * 4 | 0x20000 -- disjoint bit fields, one LOP3 after the byte's shift.
+constexpr uint32_t kClMapBase = 0x20000u;
+constexpr uint32_t kClMaxTable = kClMapBase - 1024u;  // entry-table bytes that fit below the map
 // Offset (from the start of dynamic smem) of the scratch area that follows the table.  Packed
-// tables occupy the window [0x10000, 0x20000); everything else goes above them.
+// tables occupy the window [0x10000, 0x20000); CL's class map [0x20000, 0x28000); everything else
+// goes above the table.
 __host__ __device__ constexpr uint32_t scratch_offset(int var, uint32_t table_bytes)
 {
-    return is_packed(var) ? (kPackedBase + 65536u - kSmemWindowBase) : ((table_bytes + 15u) & ~15u);
+    return is_packed(var) ? (kPackedBase + 65536u - kSmemWindowBase)
+         : var == 6 ? (kClMapBase + 256u * 128u - kSmemWindowBase)
+         : ((table_bytes + 15u) & ~15u);
 }
 __device__ __forceinline__ void check_smem_window(int var, uint32_t need)
 {
-    if (!is_packed(var)) return;
+    if (!is_packed(var) && var != 6) return;
     extern __shared__ __align__(16) uint8_t smem[];
     uint32_t dyn;
     asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(dyn));
@@ -555,29 +563,29 @@ struct TableHS {
 };
 
 // CL: byte-class compressed, lane-replicated table (DFAs with few distinct byte columns, e.g. the
-// HTML tokenizer: 38 states x 24 classes).  Class map: u32 [256][32 lanes] = shared address of the
-// lane's copy of the class row; table: u32 [N][ncls][32 lanes], entry = next * stride | count
-// (stride = ncls * 128, count in bits 0-3).  Every lookup is conflict-free (each lane reads its own
-// bank), the class lookup depends only on the input byte (off the chain), and the chain step is
-// LOP3 + IADD + LDS.32 with the count taken by one DP4A of the entry's low byte.  Chains carry the
-// entry itself (next * stride | count); ids are recovered by a multiply-high.
+// HTML tokenizer: 38 states x 24 classes).  Entry table: u32 [N][ncls][32 lanes] at the start of
+// dynamic smem, entry = next * stride | count (stride = ncls * 128, count in bits 0-3).  Class map:
+// u32 [256][32 lanes] at shared address 0x20000 = shared address of the lane's copy of the class
+// row.  Every lookup is conflict-free (each lane reads its own bank); the class-map address of
+// byte j of a word is one shift + one LOP3 ((x & 0x7F80) | 0x20000 | lane * 4), off the chain; the
+// chain step is LOP3 + IADD + LDS.32 with the count taken by one DP4A of the entry's low byte.
+// Chains carry the entry itself (next * stride | count); ids are recovered by a multiply-high.
 struct TableCL {
-    uint32_t cmbase;  // shared address of this lane's class-map column
+    uint32_t cmreg;   // kClMapBase | lane * 4
     uint32_t stride, magic;
     __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n, const KConst &kc)
     {
-        const uint32_t base = (uint32_t)__cvta_generic_to_shared(s);
+        const uint32_t tbase = (uint32_t)__cvta_generic_to_shared(s);  // 0x400 (checked)
         const uint32_t ncls = kc.ncls;
         stride = ncls * 128u;
         magic = kc.cl_magic;
         const uint32_t lane = threadIdx.x & 31;
-        cmbase = base + lane * 4;
-        const uint32_t tbase = base + 256 * 128;
+        cmreg = kClMapBase | (lane * 4);
         const uint32_t *img = static_cast<const uint32_t *>(g);
         for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
             const uint32_t c = i >> 5, l = i & 31;
             const uint32_t v = tbase + __ldg(img + c) * 128u + l * 4u;  // image: class id per byte
-            asm volatile("st.shared.u32 [%0], %1;" ::"r"(base + c * 128 + l * 4), "r"(v));
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(kClMapBase + c * 128 + l * 4), "r"(v));
         }
         for (uint32_t i = threadIdx.x; i < n * ncls * 32; i += blockDim.x) {
             const uint32_t e = i >> 5, l = i & 31;
@@ -588,12 +596,17 @@ struct TableCL {
     __device__ __forceinline__ uint32_t id_of(uint32_t cur) const { return __umulhi((cur & ~0xFu) >> 7, magic); }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return id_of(cur); }
     __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
+    // class-map address of byte j of w: the byte moved to bits 7..14, then one LOP3
+    __device__ __forceinline__ uint32_t cmaddr(uint32_t w, int j) const
+    {
+        const uint32_t x = j == 0 ? (w << 7) : (w >> (8 * j - 7));
+        return (x & 0x7F80u) | cmreg;
+    }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                          uint32_t (&accf)[K]) const
     {
-        const uint32_t c = (w >> (8 * j)) & 0xFFu;
-        const uint32_t cm = lds_u32(cmbase + (c << 7));  // class row of this lane (off the chain)
+        const uint32_t cm = lds_u32(cmaddr(w, j));  // class row of this lane (off the chain)
 #pragma unroll
         for (int s = 0; s < K; s++) {
             const uint32_t e = lds_u32((cur[s] & ~0xFu) + cm);
@@ -602,7 +615,7 @@ struct TableCL {
         }
     }
     using Row = uint32_t;
-    __device__ __forceinline__ Row row(uint32_t c) const { return lds_u32(cmbase + (c << 7)); }
+    __device__ __forceinline__ Row row(uint32_t c) const { return lds_u32(cmreg + (c << 7)); }
     __device__ __forceinline__ uint32_t apply(Row cm, uint32_t st, uint32_t &cnt) const
     {
         const uint32_t e = lds_u32(st * stride + cm);

@@ -43,7 +43,7 @@ def fits(dfa, var):
     return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "H8": n <= 8 and not dfa.bit_mode,
             "N8": n <= 8 and not dfa.bit_mode,
             "B": n <= 256, "G": True, "HS": not dfa.bit_mode and n <= 32768,
-            "CL": _n_classes(dfa) >= 2 and n * ((_n_classes(dfa) + 1) & ~1) <= 1024}[var]
+            "CL": _n_classes(dfa) >= 2 and n * ((_n_classes(dfa) + 1) & ~1) * 128 <= 0x20000 - 1024}[var]
 
 
 def _n_classes(dfa):

@@ -207,14 +207,16 @@ int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, fsm_shard_ma
  * model: every candidate's cost is its own sampled time, which already includes its sampled
  * re-execution (miss) rate.  The search is staged: (1) every instantiated k in [k_min, k_max] with the
  * default window (64 bytes, eager on) and with the paper's depth-1 look-back (eager off); (2) for
- * the two fastest k, look-back windows {0, 32, 64, 128, 256} x eager {off, 128}.
+ * the two fastest k, look-back windows {0, 32, 64, 128, 256} x eager {off, 128}; (3) for the chosen
+ * setting, every table variant the DFA fits (the by-size default is a heuristic: e.g. a random
+ * 1024-state DFA runs faster with hot-state caching, a 1027-state Aho-Corasick DFA without).
  *   input, len   device pointer and length (symbols) of the input the runs will process
  *   k_min, k_max smallest / largest k to consider (0 = 1 / min(FSM_KMAX, n_states); k_min = k_max
  *                tunes only the windows for that k)
  *   sample_len   symbols timed per candidate (0 = min(len, 2 GiB)); the prefix is used, run with the
  *                chunk and tile geometry of the full length so its cost per byte is the full run's
- *   out          the choice and its evidence; the chosen lookback_len / eager_window are also
- *                written into the handle's options (the caller passes out->k to the runs)
+ *   out          the choice and its evidence; the chosen lookback_len / eager_window / variant are
+ *                also written into the handle's options (the caller passes out->k to the runs)
  * Results of runs are identical under every setting; only speed changes.  Synchronises the
  * handle's stream.  Errors: FSM_EINVAL, FSM_ECUDA. */
 typedef struct {
@@ -226,6 +228,7 @@ typedef struct {
     double best_gbs;            /* sample bytes / median time of the chosen configuration */
     double paper_gbs;           /* same for the paper's plain setting: k = 1, depth-1 look-back, no eager */
     double hit_rate;            /* 1 - re-executed chunks / chunks, chosen configuration */
+    int32_t variant;            /* chosen table variant (FSM_VARIANT_*), applied to the options */
 } fsm_tuning;
 
 int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k_min, uint32_t k_max,

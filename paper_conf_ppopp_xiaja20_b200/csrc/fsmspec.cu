@@ -952,6 +952,7 @@ extern "C" int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, f
 namespace {
 struct TuneCand {
     uint32_t k, lookback, eager;
+    int32_t variant = FSM_VARIANT_AUTO;
     double ms = 0, hit = 0;
 };
 }  // namespace
@@ -962,6 +963,7 @@ static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom
     fsm_options o = f->opt;
     o.lookback_len = c.lookback;
     o.eager_window = c.eager;
+    o.variant = c.variant;
     o.merge = FSM_MERGE_PARALLEL;
     int rc = fsm_set_options(f, &o);
     if (rc) return rc;
@@ -969,7 +971,8 @@ static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom
     RunSpec r{nullptr, in, len, c.k, false, 0, f->start_int, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL, geom_len};
     if ((rc = launch_run(f, r))) return rc;
     if ((rc = finish_sync(f, f->d_result))) return rc;
-    c.hit = f->last.chunks ? 1.0 - (double)f->last.reexec_chunks / (double)f->last.chunks : 1.0;
+    // re-executions include the tile-candidate paths (R5), so they can exceed the chunk count
+    c.hit = f->last.chunks ? 1.0 - std::min(1.0, (double)f->last.reexec_chunks / (double)f->last.chunks) : 1.0;
     float t[3];
     for (int i = 0; i < 3; i++) {
         CK(cudaEventRecord(e0, f->stream));
@@ -1003,10 +1006,11 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
     CK(cudaEventCreate(&e1));
     std::vector<TuneCand> tried;
     int rc = FSM_OK;
-    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg) -> int {
+    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg, int32_t var = -2) -> int {
+        if (var == -2) var = saved.variant;  // stages 1-2: the handle's own variant choice
         for (const TuneCand &c : tried)
-            if (c.k == k && c.lookback == lb && c.eager == eg) return FSM_OK;
-        TuneCand c{k, lb, eg};
+            if (c.k == k && c.lookback == lb && c.eager == eg && c.variant == var) return FSM_OK;
+        TuneCand c{k, lb, eg, var};
         int r = time_candidate(f, input, n, len / sym_per_byte, c, e0, e1);
         if (r == FSM_OK) tried.push_back(c);
         return r;
@@ -1035,6 +1039,16 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
                     if (rc == FSM_OK) rc = run(k, lb, eg);
     }
     if (rc == FSM_OK) rc = run(1, 0, FSM_EAGER_OFF);  // the paper's plain spec-1, for reference
+    // stage 3: every table variant the DFA fits, at the best (k, window, eager) so far
+    if (rc == FSM_OK) {
+        const TuneCand *b = nullptr;
+        for (const TuneCand &c : tried)
+            if (c.k >= k_min && c.k <= k_max && (!b || c.ms < b->ms)) b = &c;
+        const TuneCand best_so_far = *b;
+        const int base = saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;  // what stages 1-2 ran
+        for (int v = 0; v < 8 && rc == FSM_OK; v++)
+            if (f->d_img[v] && v != base) rc = run(best_so_far.k, best_so_far.lookback, best_so_far.eager, v);
+    }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     f->opt = saved;
@@ -1054,8 +1068,11 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
     out->best_gbs = best->ms > 0 ? bytes / (best->ms * 1e6) : 0.0;
     out->paper_gbs = paper_ms > 0 ? bytes / (paper_ms * 1e6) : 0.0;
     out->hit_rate = best->hit;
+    out->variant = best->variant != FSM_VARIANT_AUTO ? best->variant
+                 : saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;
     f->opt.lookback_len = best->lookback;
     f->opt.eager_window = out->eager_window;
+    f->opt.variant = out->variant;
     return FSM_OK;
 }
 

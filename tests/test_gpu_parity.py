@@ -396,6 +396,7 @@ def test_autotune_choice_is_exact_and_not_slower():
                 assert t["k"] == kmin
             o = f.options()
             assert o["lookback_len"] == t["lookback_len"] and o["eager_window"] == t["eager_window"]
+            assert o["variant"] == t["variant"] and t["variant"] in VARIANTS.values()
             assert f.run_spec_k(ptr, data.size, t["k"]) == exp, (name, t)
         torch.cuda.synchronize()
 

@@ -58,8 +58,10 @@ enum {
                             states' rows in shared memory (u16), the rest from the u32 table in L2 */
     FSM_VARIANT_CL = 6,  /* N x byte-classes <= 1024: class-compressed, lane-replicated table, one
                             conflict-free LDS.32 per chain step (e.g. the HTML tokenizer) */
-    FSM_VARIANT_N8 = 7   /* N <= 8 (byte mode): one u32 row of eight 4-bit fields per symbol, lane-replicated
+    FSM_VARIANT_N8 = 7,  /* N <= 8 (byte mode): one u32 row of eight 4-bit fields per symbol, lane-replicated
                             smem (one LDS.32 per byte), chain = wrap-mode funnel shift + IMAD          */
+    FSM_VARIANT_R16 = 8  /* N <= 16: byte entries (next | count << 4), lane-replicated so that lane l reads
+                            bank l (128 KiB smem at N = 16), one conflict-free LDS.U8 per chain step  */
 };
 
 /* Merge strategies: the paper's parallel merge (default) and its sequential-merge baseline

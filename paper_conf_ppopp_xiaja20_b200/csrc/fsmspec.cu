@@ -52,6 +52,7 @@ FSM_DECLARE_VARIANT(g)
 FSM_DECLARE_VARIANT(hs)
 FSM_DECLARE_VARIANT(cl)
 FSM_DECLARE_VARIANT(n8)
+FSM_DECLARE_VARIANT(r16)
 
 static KernelFn get_kernel(int var, int K, bool split)
 {
@@ -62,6 +63,7 @@ static KernelFn get_kernel(int var, int K, bool split)
     case VAR_HS: return get_kernel_hs(K, split);
     case VAR_CL: return get_kernel_cl(K, split);
     case VAR_N8: return get_kernel_n8(K, split);
+    case VAR_R16: return get_kernel_r16(K, split);
     case VAR_B: return get_kernel_b(K, split);
     default: return get_kernel_g(K, split);
     }
@@ -75,6 +77,7 @@ static MultiFn get_multi(int var, int K)
     case VAR_HS: return get_multi_hs(K);
     case VAR_CL: return get_multi_cl(K);
     case VAR_N8: return get_multi_n8(K);
+    case VAR_R16: return get_multi_r16(K);
     case VAR_B: return get_multi_b(K);
     default: return get_multi_g(K);
     }
@@ -88,6 +91,7 @@ static FixFn get_fix(int var)
     case VAR_HS: return get_fix_hs();
     case VAR_CL: return get_fix_cl();
     case VAR_N8: return get_fix_n8();
+    case VAR_R16: return get_fix_r16();
     case VAR_B: return get_fix_b();
     default: return get_fix_g();
     }
@@ -101,6 +105,7 @@ static SpecFn get_spec(int var)
     case VAR_HS: return get_spec_hs();
     case VAR_CL: return get_spec_cl();
     case VAR_N8: return get_spec_n8();
+    case VAR_R16: return get_spec_r16();
     case VAR_B: return get_spec_b();
     default: return get_spec_g();
     }
@@ -114,6 +119,7 @@ static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
     case VAR_HS: get_seq_hs(K, l, w); break;
     case VAR_CL: get_seq_cl(K, l, w); break;
     case VAR_N8: get_seq_n8(K, l, w); break;
+    case VAR_R16: get_seq_r16(K, l, w); break;
     case VAR_B: get_seq_b(K, l, w); break;
     default: get_seq_g(K, l, w); break;
     }
@@ -137,8 +143,8 @@ struct fsm {
     int auto_variant = VAR_G;
     fsm_options opt{};
     // device tables
-    void *d_img[8] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
-    uint32_t img_bytes[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    void *d_img[9] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    uint32_t img_bytes[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
     uint32_t ncls = 0, cl_magic = 0;  // CL variant
     // static-frequency renumbering (hot-state caching): user <-> internal ids
     bool renumbered = false;
@@ -231,7 +237,7 @@ extern "C" int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint
 
 static void free_all(fsm *f)
 {
-    for (int i = 0; i < 8; i++) cudaFree(f->d_img[i]);
+    for (int i = 0; i < 9; i++) cudaFree(f->d_img[i]);
     cudaFree(f->d_inv);
     cudaFree(f->d_lb);
     cudaFree(f->d_nimg);
@@ -311,7 +317,9 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
     // N <= 8 in byte mode: N8 (4-bit fields, one LDS.32 per byte, batched DP4A counts) measured
     // +15..28 % over P8 (LDS.64-bound) on (8, m, k) DFAs; P4 stays ahead for N <= 4; bit mode has
     // up to 8 accepts per byte, which N8's 1-bit count field cannot hold, so it keeps P8.
-    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : (n <= 8 && !bits) ? VAR_N8 : n <= 8 ? VAR_P8 : n <= 256 ? VAR_B
+    // 8 < N <= 16: R16 (lane-replicated byte entries, conflict-free LDS.U8) measured +23..38 % over B
+    // (random-bank LDS.U16): (16, 2, k=2) 2265 -> 3034, (16, 1, k=1) 2341 -> 3224 GB/s.
+    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : (n <= 8 && !bits) ? VAR_N8 : n <= 8 ? VAR_P8 : n <= 16 ? VAR_R16 : n <= 256 ? VAR_B
                     : (f->renumbered && n > 2048) ? VAR_HS : VAR_G;
     f->opt.chunk_bytes = 0;
     f->opt.threads_per_tile = 0;  // auto: max_threads(K)
@@ -345,6 +353,11 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         auto img = image_packed(f->dfa, true);
         if ((rc = upload(&f->d_img[VAR_P8], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_P8] = 0;
+    }
+    if (n <= 16) {
+        auto img = image_r16(f->dfa);
+        if ((rc = upload(&f->d_img[VAR_R16], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_R16] = n * 8192u;  // lane-replicated in shared memory
     }
     if (n <= 256) {
         auto img = image_b(f->dfa);
@@ -425,7 +438,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
-    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_N8) return FSM_EINVAL;
+    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_R16) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
@@ -1046,7 +1059,7 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
             if (c.k >= k_min && c.k <= k_max && (!b || c.ms < b->ms)) b = &c;
         const TuneCand best_so_far = *b;
         const int base = saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;  // what stages 1-2 ran
-        for (int v = 0; v < 8 && rc == FSM_OK; v++)
+        for (int v = 0; v < 9 && rc == FSM_OK; v++)
             if (f->d_img[v] && v != base) rc = run(best_so_far.k, best_so_far.lookback, best_so_far.eager, v);
     }
     cudaEventDestroy(e0);

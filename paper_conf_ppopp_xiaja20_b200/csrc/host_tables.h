@@ -210,6 +210,15 @@ inline std::vector<uint8_t> image_n8(const ByteDFA &d)
     return img;
 }
 
+// R16 (N <= 16): byte entries E[s][c] = next | count << 4, row-major (the kernel lane-replicates
+// each u32 of four entries).
+inline std::vector<uint8_t> image_r16(const ByteDFA &d)
+{
+    std::vector<uint8_t> img((size_t)d.n * 256);
+    for (size_t i = 0; i < (size_t)d.n * 256; i++) img[i] = (uint8_t)(d.next[i] | ((uint32_t)d.inc[i] << 4));
+    return img;
+}
+
 inline std::vector<uint8_t> image_b(const ByteDFA &d)
 {
     std::vector<uint8_t> img((size_t)d.n * 512);

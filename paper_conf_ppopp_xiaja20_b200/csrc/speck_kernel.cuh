@@ -27,7 +27,7 @@
 
 namespace speck {
 
-enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5, VAR_CL = 6, VAR_N8 = 7 };
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5, VAR_CL = 6, VAR_N8 = 7, VAR_R16 = 8 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
 // in lockstep over the chunk's first kExtWindow bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
@@ -138,6 +138,12 @@ __device__ __forceinline__ uint32_t lds_u32(uint32_t a)
 {
     uint32_t v;
     asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u8(uint32_t a)
+{
+    uint32_t v;
+    asm("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
     return v;
 }
 __device__ __forceinline__ uint2 lds_v2(uint32_t a)
@@ -624,6 +630,65 @@ struct TableCL {
     }
 };
 
+// R16: N <= 16, lane-replicated byte entries E[s][c] = next | count << 4 (count 0/1 in byte mode,
+// 0..8 in bit mode).  Lane l owns bank l: the entry (s, c) of lane l sits at shared address
+//   tbase + s * 8192 + (c >> 2) * 128 + l * 4 + (c & 3)
+// (the four entries of symbols 4q..4q+3 share the lane's word), so every LDS.U8 of a warp is one
+// conflict-free wavefront whatever the lanes' states and symbols -- B's u16 table at N = 16 is read at
+// random banks (72 % replays).  128 KiB at N = 16.  The symbol part of the address is computed, not
+// loaded (two LOP3 per word, two PRMT + one IMAD per byte, off the chain); the chain step is
+// LOP3 (state bits) + IMAD (row offset) + LDS.U8.  The count of an entry is taken one step late,
+// when its state bits are masked anyway: acc += cur - (cur & 0xF) = 16 * count (one IADD3); the
+// last entry's count is still in cur when count_of runs.
+struct TableR16 {
+    uint32_t lane4;   // lane * 4 in every byte
+    uint32_t tb;      // shared address of the table (low byte 0; PRMT source of bytes 1..3)
+    uint32_t c8192, c32;
+    __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n, const KConst &kc)
+    {
+        tb = (uint32_t)__cvta_generic_to_shared(s);
+        if (tb & 0xFFu) __trap();  // the PRMT address form needs a 256-aligned table
+        lane4 = (threadIdx.x & 31) * 4u * 0x01010101u;
+        c8192 = kc.k_512 << 4;
+        c32 = kc.k_16 << 1;
+        const uint32_t *img = static_cast<const uint32_t *>(g);  // u32 [n][64]: entries 4q..4q+3 of row s
+        for (uint32_t i = threadIdx.x; i < n * 64 * 32; i += blockDim.x)
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(tb + i * 4), "r"(__ldg(img + (i >> 5))));
+    }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur & 0xFu; }
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t cur, uint64_t) const
+    {
+        return (acc >> 4) + (cur >> 4) + accf;
+    }
+    // symbol part of the address of byte j of w
+    __device__ __forceinline__ uint32_t sym(uint32_t w, int j) const
+    {
+        const uint32_t lo = (w & 0x03030303u) | lane4, hi = w & 0xFCFCFCFCu;
+        return mad_lo(prmt(hi, 0u, 0x4440u | uint32_t(j)), c32, prmt(lo, tb, 0x7650u | uint32_t(j)));
+    }
+    template <int K>
+    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
+                                         uint32_t (&accf)[K]) const
+    {
+        const uint32_t a = sym(w, j);
+#pragma unroll
+        for (int s = 0; s < K; s++) {
+            const uint32_t m = cur[s] & 0xFu;
+            acc[s] = acc[s] + cur[s] - m;          // 16 * count of the previous entry
+            cur[s] = lds_u8(mad_lo(m, c8192, a));  // next | count << 4
+        }
+    }
+    using Row = uint32_t;
+    __device__ __forceinline__ Row row(uint32_t c) const { return sym(c, 0); }
+    __device__ __forceinline__ uint32_t apply(Row a, uint32_t st, uint32_t &cnt) const
+    {
+        const uint32_t e = lds_u8(a + st * 8192u);
+        cnt += e >> 4;
+        return e & 0xFu;
+    }
+};
+
 template <int VAR> struct TableFor;
 template <> struct TableFor<VAR_P4> { using type = TablePacked<VAR_P4>; };
 template <> struct TableFor<VAR_P8> { using type = TablePacked<VAR_P8>; };
@@ -633,6 +698,7 @@ template <> struct TableFor<VAR_H8> { using type = TableH8; };
 template <> struct TableFor<VAR_HS> { using type = TableHS; };
 template <> struct TableFor<VAR_CL> { using type = TableCL; };
 template <> struct TableFor<VAR_N8> { using type = TableN8; };
+template <> struct TableFor<VAR_R16> { using type = TableR16; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <class TB> struct TableHasStep4 { static constexpr bool value = false; };
@@ -971,7 +1037,7 @@ __host__ __device__ constexpr bool split_kernel(int var, int K)
 {
     return FSM_SPLIT == 1 ? true
          : FSM_SPLIT == 0 ? false
-         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 4 || var == 2 || var == 7) /* P4 P8 H8 B N8 */ && K >= 2));
+         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 4 || var == 2 || var == 7 || var == 8) /* P4 P8 H8 B N8 R16 */ && K >= 2));
 }
 
 // Per-tile context used by re-execution and the epilogue.

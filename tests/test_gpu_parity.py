@@ -35,13 +35,13 @@ def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
     return res, st
 
 
-VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4, "HS": 5, "CL": 6, "N8": 7}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "H8": 4, "HS": 5, "CL": 6, "N8": 7, "R16": 8}
 
 
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
     return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8, "H8": n <= 8 and not dfa.bit_mode,
-            "N8": n <= 8 and not dfa.bit_mode,
+            "N8": n <= 8 and not dfa.bit_mode, "R16": n <= 16,
             "B": n <= 256, "G": True, "HS": not dfa.bit_mode and n <= 32768,
             "CL": _n_classes(dfa) >= 2 and n * ((_n_classes(dfa) + 1) & ~1) * 128 <= 0x20000 - 1024}[var]
 
@@ -70,7 +70,7 @@ def _n_classes(dfa):
 
 
 # --------------------------------------------------------------------- worked example on GPU
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "N8", "B", "G", "HS", "CL"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "N8", "R16", "B", "G", "HS", "CL"])
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
 def test_fig1_worked_example(var, k):
     d = dfas.c_comment(True)
@@ -80,7 +80,7 @@ def test_fig1_worked_example(var, k):
 
 
 # --------------------------------------------------------------------- C1-shaped text
-@pytest.mark.parametrize("var", ["P4", "P8", "H8", "N8", "B", "G", "HS", "CL"])
+@pytest.mark.parametrize("var", ["P4", "P8", "H8", "N8", "R16", "B", "G", "HS", "CL"])
 @pytest.mark.parametrize("chunk", [0, 64, 96, 4096])
 def test_c_comment_text(var, chunk):
     d = dfas.c_comment(True)
@@ -141,11 +141,28 @@ def test_div7_bits(n_bits):
     data = streams.random_bits(max(n_bits, 1), seed=n_bits)
     exp = seq.run(d, data, n_bits)
     for k in (1, 3, 7):
-        for var in ("P8", "B", "G"):
+        for var in ("P8", "B", "G", "R16"):
             got, st = gpu_run(d, data, n_bits, k=k, variant=VARIANTS[var], chunk_bytes=64)
             assert got == exp, (n_bits, k, var)
             if k == 7:
                 assert st["reexec_chunks"] == 0   # spec-N
+
+
+@pytest.mark.parametrize("n,m", [(9, 1), (12, 3), (16, 2), (16, 16)])
+@pytest.mark.parametrize("offset", [0, 5])
+def test_r16_lane_replicated_bytes(n, m, offset):
+    """R16 (N <= 16, lane-replicated byte entries): every k, both merges, look-back windows, eager
+    completion, unaligned starts and a ragged tail against the oracle."""
+    d = dfas.random_dfa(n, m, seed=7000 + n * 31 + m)
+    length = 700_001
+    data = streams.splitmix_bytes(900 + n + m, 0, length)
+    exp = seq.run(d, data)
+    for k in sorted({1, 2, 3, 4, n}):  # k <= N
+        for opt in ({}, {"merge": fsmspec.FSM_MERGE_SEQUENTIAL}, {"lookback_len": 64}, {"eager_window": 64},
+                    {"chunk_bytes": 96}):
+            got, st = gpu_run(d, data, k=k, offset=offset, variant=VARIANTS["R16"], **opt)
+            assert got == exp, (n, m, k, opt, st)
+            assert st["variant"] == VARIANTS["R16"]
 
 
 def test_div7_closed_form_on_gpu():

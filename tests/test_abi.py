@@ -128,3 +128,15 @@ def test_map_compose_vs_model_random(seed):
     mm = speck.merge(ma, mb)
     exp = [(s, e, c) for s, e, c in zip(mm.starts, mm.ends, mm.counts) if e is not None]
     assert fsmspec.map_compose(x, y).slots() == exp
+
+
+def test_variant_enum_matches_header():
+    """The binding's variant ids and names are the header's FSM_VARIANT_* enum (one table variant
+    per id; R16 = 8 is the newest)."""
+    txt = open(os.path.join(ROOT, "include", "fsmspec.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    enum = {m.group(1): int(m.group(2)) for m in re.finditer(r"FSM_VARIANT_([A-Z0-9]+)\s*=\s*(-?\d+)", txt)}
+    assert enum.pop("AUTO") == fsmspec.FSM_VARIANT_AUTO == -1
+    assert {v: k for k, v in enum.items()} == fsmspec.VARIANT_NAMES
+    for name, v in enum.items():
+        assert getattr(fsmspec, "FSM_VARIANT_" + name) == v

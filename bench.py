@@ -219,10 +219,9 @@ def certify_full(args, w, f, buf, n, k, final):
     streaming the regenerated input; the check passes iff segment 0 starts in q0, each segment
     ends where the next one claims to start, and the chained (end, count) equals the fused
     kernel's result.  By induction that is the sequential oracle over the whole input."""
-    import concurrent.futures as cf
-
     from fsmgen import streams
     from oracle import seq
+    from paper_conf_ppopp_xiaja20_b200.fsmspec import compose_from
 
     t0 = time.perf_counter()
     d = w["dfa"]
@@ -234,27 +233,15 @@ def certify_full(args, w, f, buf, n, k, final):
         claims.append(x)
         m, sh = f.run_shard(buf.data_ptr() + lo, hi - lo, halo=(buf.data_ptr() + lo - 1) if g else None,
                             halo_len=1 if g else 0, k=k, keep=True)
-        hit = [(e, c) for s, e, c in m.slots() if s == x]
-        x = hit[0][0] if hit else f.shard_fixup(sh, x)[0]
+        x2, _, miss = compose_from([m], x)
+        x = x2 if miss == 1 else f.shard_fixup(sh, x)[0]
         sh.close()
     sseed = streams.MASTER_SEED + 5
-    piece = 1 << 28
-
-    def segment(g):
-        lo, hi = bounds[g], bounds[g + 1]
-        st, total = claims[g], 0
-        tmp = np.empty(piece, dtype=np.uint8)
-        for o in range(lo, hi, piece):
-            m_ = min(piece, hi - o)
-            st, c = seq.run_from(d, st, streams.splitmix_bytes(sseed, o, m_, out=tmp), m_)
-            total += c
-        return st, total
-
-    with cf.ThreadPoolExecutor(G) as ex:
-        res = list(ex.map(segment, range(G)))
-    ok = claims[0] == d.start and all(res[g][0] == claims[g + 1] for g in range(G - 1))
-    end, total = res[-1][0], sum(c for _, c in res)
-    ok = ok and (end, total) == tuple(final)
+    try:
+        end, total = seq.certify(d, bounds, claims, lambda lo, hi: streams.splitmix_bytes(sseed, lo, hi - lo), threads=G)
+        ok = (end, total) == tuple(final)
+    except seq.CertificateError:
+        ok = False
     return {"bytes": n, "segments": G, "cores": G, "ok": bool(ok), "seconds": round(time.perf_counter() - t0, 1),
             "method": "GPU-claimed segment starts, oracle loop per segment on its own core (induction)"}
 

@@ -53,7 +53,7 @@ enum {
     FSM_VARIANT_P8 = 1,  /* N <= 8:   packed 8 x u8 row per symbol, lane-replicated smem, PRMT chain */
     FSM_VARIANT_B = 2,   /* N <= 256: u16 entries (next | count << 8) in shared memory            */
     FSM_VARIANT_G = 3,   /* any N:    u32 entries (next | count << 16) in global memory / L2      */
-    FSM_VARIANT_H8 = 4,  /* N <= 8 (byte mode): half rows of 4 states, one LDS.32 per chain step   */
+    /* 4 is retired (H8: half rows, one LDS.32 per chain step -- measured slower than P8 and N8) */
     FSM_VARIANT_HS = 5,  /* byte mode, N <= 32768: hot-state row caching (Sec. 4.2): the most frequent
                             states' rows in shared memory (u16), the rest from the u32 table in L2 */
     FSM_VARIANT_CL = 6,  /* N x byte-classes <= 1024: class-compressed, lane-replicated table, one
@@ -143,24 +143,48 @@ typedef struct {
                                    chain.  0 = default (128), FSM_EAGER_OFF = off, else 32..128 in steps
                                    of 32.  Results are identical either way; only the re-execution work
                                    changes. */
+    uint32_t preresolve;        /* delayed re-execution across tiles: a tile publishes its
+                                   aggregate mapping (one slot per speculated tile start) for the
+                                   decoupled look-back; the broken slots of the top `preresolve` start
+                                   candidates (rank order) are re-executed before publishing, so a
+                                   successor passes through them without waiting; the others are
+                                   published invalid and re-executed only if the true path enters the
+                                   tile in them.  0 = default (FSM_PRERESOLVE_DEFAULT), 1..FSM_KMAX =
+                                   top n (n >= k: every slot), FSM_PRERESOLVE_NONE = only the true path
+                                   is ever re-executed.  Results are identical under every setting. */
+    uint32_t grid_sms;          /* SMs the persistent grids use (0 = all): the grid-size sweep of the
+                                   sequential- vs parallel-merge ablation (Figs. 7-11 vary the number of
+                                   thread blocks) */
 } fsm_options;
 
 #define FSM_EAGER_OFF 1u
+#define FSM_PRERESOLVE_NONE 0x80000000u
 
 int fsm_set_options(fsm_t *f, const fsm_options *opt);
 int fsm_get_options(const fsm_t *f, fsm_options *opt);
 
-/* Counters of the most recent synchronous run on this handle (re-execution rate = reexec_chunks
- * / chunks). */
+/* Counters of the most recent run call on this handle (synchronous or asynchronous; every run
+ * call resets them, fsm_run_spec_k_host sums its pieces).  Re-execution rate = reexec_true /
+ * chunks.  "True path" = the run of the actual start state (keyed shard runs:
+ * of every valid shard slot); a8 allows re-execution only there.  Candidate-path
+ * re-executions are the optional pre-resolution of tile-start candidates (fsm_options.preresolve)
+ * that turned out not to be taken. */
 typedef struct {
     uint64_t chunks;            /* chunks processed (one thread each) */
     uint64_t tiles;             /* tiles (CTAs' work units) */
-    uint64_t reexec_chunks;     /* chunk re-executions (true-path and tile-candidate paths) */
-    uint64_t reexec_symbols;    /* bytes consumed by re-executions (early exit on convergence) */
-    uint64_t boundary_misses;   /* tile-boundary misses resolved after the look-back */
-    uint32_t chunk_bytes, threads_per_tile, variant, k_slots, lookback_len;
+    uint64_t reexec_chunks;     /* all chunk re-executions = reexec_true + reexec_candidate */
+    uint64_t reexec_symbols;    /* bytes consumed by them (early exit on convergence) */
+    uint64_t boundary_misses;   /* tile-boundary misses: true tile start not speculated */
+    uint64_t reexec_true;       /* chunk re-executions on the true path */
+    uint64_t reexec_true_symbols;
+    uint64_t reexec_candidate;  /* chunk re-executions on tile-start candidate paths not taken */
+    uint64_t reexec_candidate_symbols;
+    uint64_t eager_resolved;    /* true-path misses completed from an eager-completion entry (NEXT-3) */
+    uint64_t max_miss_chain;    /* longest run of consecutive re-executed chunks on the true path */
+    uint32_t chunk_bytes, threads_per_tile, variant, k_slots, lookback_len, preresolve;
 } fsm_stats;
 
+/* Synchronises the handle's stream (the counters live on the device). */
 int fsm_get_stats(const fsm_t *f, fsm_stats *s);
 
 /* ---------------------------------------------------------------- shard level (multi-GPU) ---
@@ -177,14 +201,15 @@ typedef struct {
 
 typedef struct fsm_shard fsm_shard_t;  /* per-shard state kept for a later fix-up */
 
-/* fsm_run_shard: run one shard.
+/* fsm_run_shard: run one shard.  An out-of-alphabet byte inside the shard drives every path into
+ * the sink, so it is reported as FSM_ESYMBOL here (no map is written).
  *   input, len  device pointer and length (bytes, or bits in bit mode; bit-mode shards must start
  *               on a byte boundary, i.e. every shard but the last has len % 8 == 0).
  *   halo        device pointer to the halo_len bytes immediately before the shard, or NULL with
  *               halo_len = 0 for shard 0 (start = q0).  Only the last halo byte is used.
  *   out         receives the mapping; state (optional) receives a handle for fsm_shard_fixup,
  *               which borrows `input` until fsm_shard_free.
- * Errors: FSM_EINVAL, FSM_ECUDA, FSM_ENOMEM. */
+ * Errors: FSM_EINVAL, FSM_ESYMBOL, FSM_ECUDA, FSM_ENOMEM. */
 int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const uint8_t *halo,
                   uint32_t halo_len, uint32_t k, fsm_shard_map *out, fsm_shard_t **state);
 
@@ -200,6 +225,17 @@ void fsm_shard_free(fsm_shard_t *state);  /* NULL is a no-op */
  * whose end is a start of b continues with b's end and adds counts; otherwise it becomes invalid
  * (delayed strategy).  out may alias a or b. */
 int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, fsm_shard_map *out);
+
+/* fsm_compose_from: host-only, pure.  Follows the state `start_state` (count `start_count`) through
+ * maps[0 .. n) in order -- at each map, the valid slot whose start equals the current state gives
+ * the next state and adds its count (the membership check of Alg. 1, applied to shard
+ * maps, SURVEY.md 8.e "Compose").  Stops at the first map with no such slot: *first_miss = its
+ * index (that shard's true start was not speculated; the caller runs fsm_shard_fixup there and
+ * continues from map first_miss + 1), or n when every map matched.  *state / *count are the state
+ * and count before maps[*first_miss] (after the last map when *first_miss == n).
+ * Errors: FSM_EINVAL (NULL pointers with n > 0). */
+int fsm_compose_from(const fsm_shard_map *maps, uint32_t n, uint32_t start_state, uint64_t start_count,
+                     uint32_t *state, uint64_t *count, uint32_t *first_miss);
 
 /* ------------------------------------------------------------- NEXT-2: k / look-back tuning ---
  * The paper leaves the choice of k to the user and names a cost model for it as future work
@@ -264,6 +300,38 @@ int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *input, uint64_t
  * min(|image|, FSM_KMAX).  States are internal ids (the sink, if any, is id n_states). */
 int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint32_t alphabet,
                        uint32_t input_mode, uint16_t *lb_out, uint8_t *nimg_out);
+
+/* ---------------------------------------------------------------------- test-only hooks ---
+ * Used by tests to replay the paper's worked examples on the CUDA merge (Fig. 2; Fig. 4,
+ * P:103-105; SURVEY.md 8.b "Python layer" and 8.c.3 P2-P4).  Not for production use.
+ *
+ * fsm_debug_set_spec: fix the geometry of the following runs on f to chunks of `chunk_bytes` bytes
+ * (1 .. 8192, any value) in tiles of 32 chunks, and -- if `sets` is not NULL -- inject the
+ * speculated start sets: sets[j * k + s] = slot s of chunk j (user state ids, 0xFFFFFFFF = no
+ * state), for chunks 0 .. n_chunks-1, chunk 0 included (this overrides reading A7's S_0 = {q0};
+ * the true start must then be one of chunk 0's slots or is resolved by re-execution like any
+ * miss).  Runs must have exactly n_chunks chunks and the same k.  The look-back window and eager
+ * completion are off while injected.  chunk_bytes = 0 clears everything.
+ * Errors: FSM_EINVAL (k out of range, a state >= n_states, n_chunks = 0 with sets). */
+int fsm_debug_set_spec(fsm_t *f, const uint32_t *sets, uint32_t n_chunks, uint32_t k, uint32_t chunk_bytes);
+
+/* The merge tree of tile 0, warp 0 of the most recent run made under fsm_debug_set_spec: level 0 =
+ * each chunk's own mapping M_j (lane j), level l = lane j's mapping after the l-th warp-scan level,
+ * i.e. M_j x ... x M_{j + 2^l - 1} (Fig. 4b: level 1 lane 0 = chunks 0+1, lane 2 = chunks 2+3,
+ * level 2 lane 0 = the root).  Slot s of lane j at level l: start = speculated start of chunk j
+ * (0xFFFFFFFF = none); valid = the slot's run passed every membership check so far;
+ * end / count = the state reached and F-visits (meaningful when valid; when invalid, end = the
+ * state at the chunk where the check failed and brk = that chunk's index).  States in user ids. */
+typedef struct {
+    uint32_t k;                              /* slots per mapping (the run's instantiated K) */
+    uint32_t start[6][32][FSM_KMAX];
+    uint32_t end[6][32][FSM_KMAX];
+    uint32_t count[6][32][FSM_KMAX];
+    uint32_t brk[6][32][FSM_KMAX];           /* 0xFFFFFFFF = valid; 0xFFFFFFFE = no state */
+    uint32_t identity[6][32];                /* lane held no chunk (past the end of the input) */
+} fsm_debug_merge;
+
+int fsm_debug_get_merge(const fsm_t *f, fsm_debug_merge *out);
 
 /* Library version string. */
 const char *fsm_version(void);

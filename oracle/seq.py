@@ -3,7 +3,6 @@
 run(dfa, data, length)          -> (final_state, accept_count)   C loop, any size
 run_py(table, start, F, syms)   -> same, pure Python (tiny cases; pins the C loop)
 run_from(...)                   -> from an arbitrary start state (used for shard maps / certificates)
-run_splitmix(dfa, seed, length) -> streams the counter-based C5 input through the C loop
 certify(...)                    -> multi-core check of claimed segment start states
 Definition: q_i = delta(q_{i-1}, x_i), count = |{i in [1, L] : q_i in F}| (readings A3, A4).
 """
@@ -93,47 +92,36 @@ def bits_of(data: np.ndarray, n_bits: int) -> list[int]:
     return [int((int(data[i >> 3]) >> (7 - (i & 7))) & 1) for i in range(n_bits)]
 
 
-def run_splitmix(dfa, seed: int, length: int, start: int | None = None, offset: int = 0,
-                 piece: int = 1 << 28) -> tuple[int, int]:
-    """Stream bytes [offset, offset+length) of the counter-based generator through the loop,
-    piece by piece (the generator regenerates the bytes the GPU side generated in place)."""
-    from fsmgen import streams
-
-    q = dfa.start if start is None else start
-    cnt = 0
-    cache = _arrays(dfa)
-    buf = np.empty(min(piece, max(length, 1)), dtype=np.uint8)
-    pos = 0
-    while pos < length:
-        n = min(piece, length - pos)
-        streams.splitmix_bytes(seed, offset + pos, n, out=buf)
-        q, c = run_from(dfa, q, buf[:n], n, _cache=cache)
-        cnt += c
-        pos += n
-    return q, cnt
+class CertificateError(AssertionError):
+    """The GPU-claimed segment start states are not the oracle's."""
 
 
-def certify(dfa, segments: list[tuple[int, int]], claimed_starts: list[int], fetch,
+def certify(dfa, bounds: list[int], claimed_starts: list[int], fetch, piece: int = 1 << 28,
             threads: int | None = None) -> tuple[int, int]:
-    """Certificate check.  ``segments`` = contiguous [lo, hi) byte ranges that
-    tile [0, L); ``claimed_starts[i]`` = the state the GPU claims at ``segments[i][0]``;
-    ``fetch(lo, hi)`` returns those input bytes.  Each segment runs the plain loop from its claimed
-    start on its own core; the check passes only if segment 0 starts at q0 and every segment ends
-    where the next one claims to start.  By induction the result equals the sequential oracle."""
-    assert segments and segments[0][0] == 0
+    """Certificate check of a long byte-mode run.  ``bounds`` = b_0 = 0 < b_1 <
+    ... < b_G = L cut the input into G contiguous segments; ``claimed_starts[g]`` = the state a
+    GPU run claims at b_g; ``fetch(lo, hi)`` returns input bytes [lo, hi) (called piece by piece,
+    so inputs far larger than host memory stream through).  Every segment runs the plain loop
+    (``run_from``) from its claimed start, on its own thread; the check passes only if segment 0
+    starts in q0 and every segment ends where the next one claims to start -- then, by induction
+    over the segments, the concatenation is the sequential run of Fig. 1c over the whole input and
+    the returned (final state, summed count) is the oracle's result.  Raises CertificateError."""
+    assert not dfa.bit_mode and len(bounds) == len(claimed_starts) + 1 and bounds[0] == 0
     if claimed_starts[0] != dfa.start:
-        raise AssertionError("segment 0 does not start at q0")
+        raise CertificateError(f"segment 0 claims {claimed_starts[0]}, q0 = {dfa.start}")
     cache = _arrays(dfa)
 
-    def one(i):
-        lo, hi = segments[i]
-        return run_from(dfa, claimed_starts[i], fetch(lo, hi), hi - lo, _cache=cache)
+    def one(g):
+        q, total = claimed_starts[g], 0
+        for o in range(bounds[g], bounds[g + 1], piece):
+            hi = min(o + piece, bounds[g + 1])
+            q, c = run_from(dfa, q, fetch(o, hi), hi - o, _cache=cache)
+            total += c
+        return q, total
 
-    with cf.ThreadPoolExecutor(max_workers=threads or os.cpu_count()) as ex:
-        res = list(ex.map(one, range(len(segments))))
-    total = 0
-    for i, (end, c) in enumerate(res):
-        total += c
-        if i + 1 < len(segments) and end != claimed_starts[i + 1]:
-            raise AssertionError(f"segment {i} ends in {end}, next claims {claimed_starts[i + 1]}")
-    return res[-1][0], total
+    with cf.ThreadPoolExecutor(max_workers=threads or min(len(claimed_starts), os.cpu_count() or 1)) as ex:
+        res = list(ex.map(one, range(len(claimed_starts))))
+    for g in range(len(res) - 1):
+        if res[g][0] != claimed_starts[g + 1]:
+            raise CertificateError(f"segment {g} ends in {res[g][0]}, segment {g + 1} claims {claimed_starts[g + 1]}")
+    return res[-1][0], sum(c for _, c in res)

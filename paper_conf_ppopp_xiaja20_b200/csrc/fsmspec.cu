@@ -46,7 +46,6 @@ typedef void (*MultiFn)(Params, const Params *, uint32_t);
     SpecFn get_spec_##NAME();
 FSM_DECLARE_VARIANT(p4)
 FSM_DECLARE_VARIANT(p8)
-FSM_DECLARE_VARIANT(h8)
 FSM_DECLARE_VARIANT(b)
 FSM_DECLARE_VARIANT(g)
 FSM_DECLARE_VARIANT(hs)
@@ -59,7 +58,6 @@ static KernelFn get_kernel(int var, int K, bool split)
     switch (var) {
     case VAR_P4: return get_kernel_p4(K, split);
     case VAR_P8: return get_kernel_p8(K, split);
-    case VAR_H8: return get_kernel_h8(K, split);
     case VAR_HS: return get_kernel_hs(K, split);
     case VAR_CL: return get_kernel_cl(K, split);
     case VAR_N8: return get_kernel_n8(K, split);
@@ -73,7 +71,6 @@ static MultiFn get_multi(int var, int K)
     switch (var) {
     case VAR_P4: return get_multi_p4(K);
     case VAR_P8: return get_multi_p8(K);
-    case VAR_H8: return get_multi_h8(K);
     case VAR_HS: return get_multi_hs(K);
     case VAR_CL: return get_multi_cl(K);
     case VAR_N8: return get_multi_n8(K);
@@ -87,7 +84,6 @@ static FixFn get_fix(int var)
     switch (var) {
     case VAR_P4: return get_fix_p4();
     case VAR_P8: return get_fix_p8();
-    case VAR_H8: return get_fix_h8();
     case VAR_HS: return get_fix_hs();
     case VAR_CL: return get_fix_cl();
     case VAR_N8: return get_fix_n8();
@@ -101,7 +97,6 @@ static SpecFn get_spec(int var)
     switch (var) {
     case VAR_P4: return get_spec_p4();
     case VAR_P8: return get_spec_p8();
-    case VAR_H8: return get_spec_h8();
     case VAR_HS: return get_spec_hs();
     case VAR_CL: return get_spec_cl();
     case VAR_N8: return get_spec_n8();
@@ -115,7 +110,6 @@ static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
     switch (var) {
     case VAR_P4: get_seq_p4(K, l, w); break;
     case VAR_P8: get_seq_p8(K, l, w); break;
-    case VAR_H8: get_seq_h8(K, l, w); break;
     case VAR_HS: get_seq_hs(K, l, w); break;
     case VAR_CL: get_seq_cl(K, l, w); break;
     case VAR_N8: get_seq_n8(K, l, w); break;
@@ -179,9 +173,12 @@ struct fsm {
     // sequential-merge ablation buffers
     SeqBuf seq{};
     size_t seq_cap = 0;
-    // stats of the last synchronous run
+    // geometry / configuration of the most recent run (the counters are read from d_stats)
     fsm_stats last{};
-    DevStats stats_before{};
+    // test hook (fsm_debug_set_spec): fixed chunk bytes, injected sets, merge-tree readback
+    uint32_t dbg_chunk = 0, dbg_n = 0, dbg_k = 0;
+    uint16_t *d_dbg_spec = nullptr;
+    uint4 *d_dbg = nullptr;
     // hex lookback for host queries
     std::vector<uint16_t> lb;
     std::vector<uint8_t> nimg;
@@ -191,6 +188,7 @@ struct fsm_shard {
     const uint8_t *input = nullptr;
     uint64_t len = 0;          // symbols
     uint32_t k = 0;
+    int variant = 0;           // the table variant the shard ran with (the fix-up uses the same)
     fsm_shard_map map{};
 };
 
@@ -251,6 +249,8 @@ static void free_all(fsm *f)
     cudaFree(f->d_stage[1]);
     cudaFree(f->d_spec);
     cudaFree(f->d_multi);
+    cudaFree(f->d_dbg_spec);
+    cudaFree(f->d_dbg);
     cudaFree(f->seq.S);
     cudaFree(f->seq.E);
     cudaFree(f->seq.C);
@@ -338,11 +338,6 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         auto img = image_packed(f->dfa, false);
         if ((rc = upload(&f->d_img[VAR_P4], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_P4] = 0;  // packed tables live in a fixed shared-window slot (scratch_offset)
-    }
-    if (n <= 8 && !bits) {  // H8's count bit is byte-mode only
-        auto img = image_h8(f->dfa);
-        if ((rc = upload(&f->d_img[VAR_H8], img.data(), img.size()))) return fail(rc);
-        f->img_bytes[VAR_H8] = 0;
     }
     if (n <= 8 && !bits) {  // N8's count bit is byte-mode only
         auto img = image_n8(f->dfa);
@@ -439,17 +434,20 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
     if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_R16) return FSM_EINVAL;
-    if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // table too large for it
+    if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // too large, or retired (4)  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
     if (o->eager_window > FSM_EAGER_OFF && (o->eager_window % 32 || o->eager_window > kExtWindow)) return FSM_EINVAL;
+    if (o->preresolve > FSM_KMAX && o->preresolve != FSM_PRERESOLVE_NONE) return FSM_EINVAL;
     f->opt.chunk_bytes = o->chunk_bytes;            // 0 = adaptive
     f->opt.threads_per_tile = o->threads_per_tile;  // 0 = auto
     f->opt.variant = o->variant;
     f->opt.merge = o->merge;
     f->opt.ctas_per_sm = o->ctas_per_sm;
+    f->opt.grid_sms = o->grid_sms;
     f->opt.lookback_len = o->lookback_len;
     f->opt.eager_window = o->eager_window;
+    f->opt.preresolve = o->preresolve;
     return FSM_OK;
 }
 
@@ -463,7 +461,20 @@ extern "C" int fsm_get_options(const fsm_t *f, fsm_options *o)
 extern "C" int fsm_get_stats(const fsm_t *f, fsm_stats *s)
 {
     if (!f || !s) return FSM_EINVAL;
-    *s = f->last;
+    DevStats h{};
+    CK(cudaMemcpyAsync(&h, f->d_stats, sizeof(DevStats), cudaMemcpyDeviceToHost, f->stream));
+    CK(cudaStreamSynchronize(f->stream));
+    fsm_stats r = f->last;
+    r.reexec_true = h.reexec_true;
+    r.reexec_true_symbols = h.reexec_true_bytes;
+    r.reexec_candidate = h.reexec_cand;
+    r.reexec_candidate_symbols = h.reexec_cand_bytes;
+    r.reexec_chunks = h.reexec_true + h.reexec_cand;
+    r.reexec_symbols = h.reexec_true_bytes + h.reexec_cand_bytes;
+    r.boundary_misses = h.boundary_misses;
+    r.eager_resolved = h.eager_resolved;
+    r.max_miss_chain = h.max_miss_chain;
+    *s = r;
     return FSM_OK;
 }
 
@@ -483,7 +494,16 @@ struct RunSpec {
     uint64_t geom_len_bytes = 0;  // geometry as for a run of this many bytes (0 = len): tuning samples
     uint32_t force_T = 0, force_chunk = 0;  // multi-FSM groups: one geometry for every DFA
     bool multi = false;                     // launched by the multi-FSM kernel (never split)
+    bool accumulate = false;                // keep the counters of the call's earlier launches
 };
+
+// R5 default (fsm_options.preresolve = 0): see DESIGN.md "R5".
+constexpr uint32_t kPreresolveDefault = FSM_KMAX;
+static uint32_t preresolve_of(const fsm *f)
+{
+    const uint32_t v = f->opt.preresolve;
+    return v == 0 ? kPreresolveDefault : v == FSM_PRERESOLVE_NONE ? 0u : v;
+}
 
 // Chunks per tile: a split kernel (split_kernel(var, K)) gives the CTA's last warp to the epilogue.
 static uint32_t tile_chunks(uint32_t T, bool split) { return split ? T - 32 : T; }
@@ -493,9 +513,6 @@ static int variant_of(const fsm *f, int force, uint32_t k = 1)
 {
     if (force >= 0) return force;
     if (f->opt.variant != FSM_VARIANT_AUTO) return f->opt.variant;
-    // H8 (one LDS.32 per chain step, on the dependency chain) measured slower than P8 (one LDS.64
-    // per byte, off the chain) on B200: 3.21 vs 3.73 TB/s at k = 1, so the
-    // automatic choice keeps P8; H8 stays selectable.
     (void)k;
     return f->auto_variant;
 }
@@ -534,6 +551,12 @@ static int ensure_desc(fsm *f, size_t ntiles)
 }
 
 static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T);
+// SMs the persistent grids are spread over (fsm_options.grid_sms; the a11 grid-size sweep)
+static uint64_t grid_sms(const fsm *f)
+{
+    return f->opt.grid_sms ? std::min<uint64_t>(f->opt.grid_sms, (uint64_t)f->num_sms) : (uint64_t)f->num_sms;
+}
+constexpr size_t kDbgBytes = (size_t)6 * 32 * KMAX * sizeof(uint4);  // fsm_debug_get_merge levels
 
 // Everything of a run but the fused kernel's launch: variant, geometry, Params, the look-back
 // pre-pass (launched here), descriptors.  Shared by single runs and multi-FSM groups.
@@ -550,11 +573,31 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     const int var = variant_of(f, r.force_variant, r.k);
     const int K = kslots(r.k);
     const bool bits = f->mode == FSM_INPUT_BITS_MSB;
-    const uint64_t len_bytes = bits ? r.len_sym / 8 : r.len_sym;
+    const uint64_t ulen_bytes = bits ? r.len_sym / 8 : r.len_sym;
+    // An unaligned input is run from the 32-byte-aligned address below it: chunk 0 is [head, chunk)
+    // and every kernel position is relative to that address, so every other chunk starts on a full
+    // sector (one peeled partial sector instead of a byte-at-a-time run).  Debug geometries with
+    // tiny chunks on an unaligned input keep the byte path instead.
+    uint32_t head = (uint32_t)((uintptr_t)r.in & 31);
+    bool aligned = true;
+    if (head && f->dbg_chunk && !r.multi && f->dbg_chunk < 64) {
+        head = 0;
+        aligned = false;
+    }
+    const uint64_t len_bytes = ulen_bytes + head;  // kernel coordinates
     uint32_t T = 0, chunk = 0;
-    pick_geometry(f, r.geom_len_bytes ? std::max(r.geom_len_bytes, len_bytes) : len_bytes, K, T, chunk);
+    pick_geometry(f, r.geom_len_bytes ? std::max(r.geom_len_bytes, ulen_bytes) : ulen_bytes, K, T, chunk);
     if (r.force_T) T = r.force_T;
     if (r.force_chunk) chunk = r.force_chunk;
+    const bool dbg = f->dbg_chunk != 0 && !r.multi;
+    if (dbg) {  // test hook: the fixed tiny geometry of fsm_debug_set_spec (one warp of chunks per tile)
+        chunk = f->dbg_chunk;
+        T = 32;
+        if (f->dbg_n) {
+            const uint64_t nch = len_bytes == 0 ? 1 : (len_bytes + chunk - 1) / chunk;
+            if (nch != f->dbg_n || r.k != f->dbg_k || r.keyed || head) return FSM_EINVAL;
+        }
+    }
     if (r.merge == FSM_MERGE_SEQUENTIAL) T = std::min<uint32_t>(T, kThreads);
     if (split_kernel(var, K) && T < 64) T = 64;  // at least one worker warp besides the epilogue warp
     bool split = split_kernel(var, K) && !r.multi && r.merge == FSM_MERGE_PARALLEL;
@@ -570,14 +613,27 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     int rc;
 
     Params p{};
-    p.in = r.in;
+    p.in = r.in - head;
+    p.head = head;
     p.len = len_bytes;
     p.chunk = chunk;
     p.ntiles = ntiles;
     p.k = r.k;
     p.lookback = f->opt.lookback_len > 1 ? f->opt.lookback_len : 0;
     p.eager_window = f->opt.eager_window == 0 ? kExtWindow : f->opt.eager_window == FSM_EAGER_OFF ? 0u : f->opt.eager_window;
-    p.aligned = ((uintptr_t)r.in & 31) == 0;
+    p.preresolve = preresolve_of(f);
+    if (dbg && f->dbg_n) {
+        p.lookback = 0;
+        p.eager_window = 0;
+        p.spec = f->d_dbg_spec;
+        p.spec_stride = r.k + kExt;
+        p.spec_all = 1;
+    }
+    if (dbg) {
+        p.dbg = f->d_dbg;
+        CK(cudaMemsetAsync(f->d_dbg, 0xFF, kDbgBytes, f->stream));
+    }
+    p.aligned = aligned ? 1u : 0u;
     p.table = f->d_img[var];
     p.n_states = f->dfa.n;
     p.table_bytes = f->img_bytes[var];
@@ -660,11 +716,13 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     f->last.variant = var;
     f->last.k_slots = K;
     f->last.lookback_len = p.lookback;
+    f->last.preresolve = p.preresolve;
     return FSM_OK;
 }
 
 static int launch_run(fsm *f, const RunSpec &r)
 {
+    if (!r.accumulate) CK(cudaMemsetAsync(f->d_stats, 0, sizeof(DevStats), f->stream));  // per-call counters
     Prepared pr;
     int rc = prepare_run(f, r, pr);
     if (rc) return rc;
@@ -684,7 +742,7 @@ static int launch_run(fsm *f, const RunSpec &r)
     if (occ < 1) return FSM_EINVAL;
     if (f->opt.ctas_per_sm) occ = std::min<int>(occ, (int)f->opt.ctas_per_sm);
     const uint32_t ntiles = p.ntiles;
-    const uint32_t grid = (uint32_t)std::min<uint64_t>(ntiles, (uint64_t)occ * f->num_sms);
+    const uint32_t grid = (uint32_t)std::min<uint64_t>(ntiles, (uint64_t)occ * grid_sms(f));
     p.ticket_base = f->ticket_base;
     fn<<<grid, T, smem, f->stream>>>(p);
     CK(cudaGetLastError());
@@ -715,7 +773,7 @@ static int launch_seq(fsm *f, Params p, int var, int K, uint32_t T)
     CK(cudaFuncSetAttribute((const void *)lf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(smem_l, 16)));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lf, (int)T, std::max<size_t>(smem_l, 16)));
-    const uint64_t blocks = std::min<uint64_t>((nch + T - 1) / T, (uint64_t)std::max(occ, 1) * f->num_sms);
+    const uint64_t blocks = std::min<uint64_t>((nch + T - 1) / T, (uint64_t)std::max(occ, 1) * grid_sms(f));
     lf<<<(uint32_t)blocks, T, std::max<size_t>(smem_l, 16), f->stream>>>(p, f->seq);
     CK(cudaGetLastError());
     const size_t smem_w = seq_walk_smem(T, K, var, p.table_bytes);
@@ -740,18 +798,11 @@ static int check_run_args(const fsm *f, const uint8_t *input, uint64_t len, uint
     return FSM_OK;
 }
 
-// Read result + stats of the run just enqueued (one small D2H), fill f->last.
+// Read the result of the run just enqueued (one small D2H).
 static int finish_sync(fsm *f, const DevResult *dres)
 {
-    DevResult *hr = f->h_result;
-    DevStats *hs = reinterpret_cast<DevStats *>(hr + 1);
-    CK(cudaMemcpyAsync(hr, dres, sizeof(DevResult), cudaMemcpyDeviceToHost, f->stream));
-    CK(cudaMemcpyAsync(hs, f->d_stats, sizeof(DevStats), cudaMemcpyDeviceToHost, f->stream));
+    CK(cudaMemcpyAsync(f->h_result, dres, sizeof(DevResult), cudaMemcpyDeviceToHost, f->stream));
     CK(cudaStreamSynchronize(f->stream));
-    f->last.reexec_chunks = hs->reexec_chunks - f->stats_before.reexec_chunks;
-    f->last.reexec_symbols = hs->reexec_bytes - f->stats_before.reexec_bytes;
-    f->last.boundary_misses = hs->boundary_misses - f->stats_before.boundary_misses;
-    f->stats_before = *hs;
     return FSM_OK;
 }
 
@@ -822,6 +873,7 @@ extern "C" int fsm_run_spec_k_host(fsm_t *f, const uint8_t *host_input, uint64_t
         DevResult *res = f->d_result + ((pi + 1) & 1);
         const DevResult *prev = pi == 0 ? nullptr : f->d_result + (pi & 1);
         RunSpec r{nullptr, f->d_stage[sb], sym, k, false, 0, f->start_int, prev, res, -1, FSM_MERGE_PARALLEL};
+        r.accumulate = pi > 0;  // the call's counters sum over its pieces
         if ((rc = launch_run(f, r))) return rc;
         CK(cudaEventRecord(f->ev_used[sb], f->stream));
         chunks += f->last.chunks;
@@ -856,6 +908,11 @@ extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const
     if ((rc = launch_run(f, r))) return rc;
     if ((rc = finish_sync(f, f->d_result))) return rc;
     const DevResult *hr = f->h_result;
+    // an out-of-alphabet byte maps every state to the absorbing sink: every path ends there
+    if (!keyed && is_sink(f, hr->final_state)) return FSM_ESYMBOL;
+    if (keyed)
+        for (int s = 0; s < KMAX; s++)
+            if (((hr->valid_mask >> s) & 1u) && is_sink(f, hr->end[s])) return FSM_ESYMBOL;
     fsm_shard_map m{};
     m.k = k;
     if (!keyed) {
@@ -879,6 +936,7 @@ extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const
         st->input = input;
         st->len = len;
         st->k = k;
+        st->variant = (int)f->last.variant;
         st->map = m;
         *state = st;
     }
@@ -896,7 +954,7 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         }
     const bool bits = f->mode == FSM_INPUT_BITS_MSB;
     const uint64_t whole = bits ? st->len / 8 : st->len;
-    const int var = variant_of(f, -1);
+    const int var = st->variant;
     FixParams fp{};
     fp.in = st->input;
     fp.len = whole;
@@ -929,7 +987,7 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         return FSM_OK;
     }
     // no convergence: exact parallel re-run of the shard from the true start
-    RunSpec r{nullptr, st->input, st->len, st->k, false, 0, to_int(f, true_start), nullptr, f->d_result, -1,
+    RunSpec r{nullptr, st->input, st->len, st->k, false, 0, to_int(f, true_start), nullptr, f->d_result, var,
               FSM_MERGE_PARALLEL};
     int rc = launch_run(f, r);
     if (rc) return rc;
@@ -940,6 +998,70 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
 }
 
 extern "C" void fsm_shard_free(fsm_shard_t *st) { delete st; }
+
+// ---------------------------------------------------------------------------- test hooks ----
+extern "C" int fsm_debug_set_spec(fsm_t *f, const uint32_t *sets, uint32_t n_chunks, uint32_t k, uint32_t chunk_bytes)
+{
+    if (!f) return FSM_EINVAL;
+    if (chunk_bytes == 0) {
+        f->dbg_chunk = f->dbg_n = f->dbg_k = 0;
+        return FSM_OK;
+    }
+    if (chunk_bytes > 8192) return FSM_EINVAL;
+    if (sets) {
+        if (n_chunks == 0 || k < 1 || k > FSM_KMAX || k > f->n_user) return FSM_EINVAL;
+        const uint32_t stride = k + kExt;
+        std::vector<uint16_t> h((size_t)n_chunks * stride, 0xFFFFu);
+        for (uint32_t j = 0; j < n_chunks; j++)
+            for (uint32_t s = 0; s < k; s++) {
+                const uint32_t v = sets[(size_t)j * k + s];
+                if (v == 0xFFFFFFFFu) continue;
+                if (v >= f->n_user) return FSM_EINVAL;
+                for (uint32_t q = 0; q < s; q++)
+                    if (sets[(size_t)j * k + q] == v) return FSM_EINVAL;  // reading A6: never duplicated
+                h[(size_t)j * stride + s] = (uint16_t)to_int(f, v);
+            }
+        cudaStreamSynchronize(f->stream);
+        cudaFree(f->d_dbg_spec);
+        f->d_dbg_spec = nullptr;
+        int rc = upload(&f->d_dbg_spec, h.data(), h.size() * 2);
+        if (rc) return rc;
+    }
+    if (!f->d_dbg) CK(cudaMalloc(&f->d_dbg, kDbgBytes));
+    f->dbg_chunk = chunk_bytes;
+    f->dbg_n = sets ? n_chunks : 0;
+    f->dbg_k = sets ? k : 0;
+    return FSM_OK;
+}
+
+extern "C" int fsm_debug_get_merge(const fsm_t *f, fsm_debug_merge *out)
+{
+    if (!f || !out || !f->d_dbg) return FSM_EINVAL;
+    std::vector<uint4> h(kDbgBytes / sizeof(uint4));
+    CK(cudaStreamSynchronize(f->stream));
+    CK(cudaMemcpy(h.data(), f->d_dbg, kDbgBytes, cudaMemcpyDeviceToHost));
+    const uint32_t K = f->last.k_slots;
+    out->k = K;
+    for (int l = 0; l < 6; l++)
+        for (int lane = 0; lane < 32; lane++) {
+            out->identity[l][lane] = h[(size_t)(l * 32 + lane) * KMAX].w == 1u;
+            for (uint32_t s = 0; s < (uint32_t)KMAX; s++) {
+                const uint4 v = h[(size_t)(l * 32 + lane) * KMAX + s];
+                const uint32_t code = v.y >> 16, st = v.y & 0xFFFFu;
+                const bool have = s < K && v.x != NOSTATE && v.x != 0xFFFFFFFFu;
+                out->start[l][lane][s] = have ? to_user(f, v.x) : 0xFFFFFFFFu;
+                out->count[l][lane][s] = have ? v.z : 0u;
+                if (!have || code == ABSENT) {
+                    out->brk[l][lane][s] = 0xFFFFFFFEu;
+                    out->end[l][lane][s] = 0xFFFFFFFFu;
+                } else {
+                    out->brk[l][lane][s] = code == COMPLETE ? 0xFFFFFFFFu : code;
+                    out->end[l][lane][s] = to_user(f, st);
+                }
+            }
+        }
+    return FSM_OK;
+}
 
 extern "C" int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, fsm_shard_map *out)
 {
@@ -957,6 +1079,28 @@ extern "C" int fsm_map_compose(const fsm_shard_map *a, const fsm_shard_map *b, f
             }
     }
     *out = r;
+    return FSM_OK;
+}
+
+extern "C" int fsm_compose_from(const fsm_shard_map *maps, uint32_t n, uint32_t start_state, uint64_t start_count,
+                                uint32_t *state, uint64_t *count, uint32_t *first_miss)
+{
+    if (!state || !count || !first_miss || (n > 0 && !maps)) return FSM_EINVAL;
+    uint32_t x = start_state;
+    uint64_t c = start_count;
+    uint32_t g = 0;
+    for (; g < n; g++) {
+        const fsm_shard_map &m = maps[g];
+        int hit = -1;
+        for (int s = 0; s < KMAX && hit < 0; s++)
+            if (((m.valid_mask >> s) & 1u) && m.start[s] == x) hit = s;
+        if (hit < 0) break;
+        x = m.end[hit];
+        c += m.count[hit];
+    }
+    *state = x;
+    *count = c;
+    *first_miss = g;
     return FSM_OK;
 }
 
@@ -984,8 +1128,9 @@ static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom
     RunSpec r{nullptr, in, len, c.k, false, 0, f->start_int, nullptr, f->d_result, -1, FSM_MERGE_PARALLEL, geom_len};
     if ((rc = launch_run(f, r))) return rc;
     if ((rc = finish_sync(f, f->d_result))) return rc;
-    // re-executions include the tile-candidate paths (R5), so they can exceed the chunk count
-    c.hit = f->last.chunks ? 1.0 - std::min(1.0, (double)f->last.reexec_chunks / (double)f->last.chunks) : 1.0;
+    fsm_stats st;
+    if ((rc = fsm_get_stats(f, &st))) return rc;
+    c.hit = st.chunks ? 1.0 - (double)st.reexec_true / (double)st.chunks : 1.0;
     float t[3];
     for (int i = 0; i < 3; i++) {
         CK(cudaEventRecord(e0, f->stream));
@@ -1127,6 +1272,11 @@ extern "C" int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *inpu
         }
         lead->multi_cap = m;
     }
+    for (uint32_t i = 0; i < m; i++)  // per-call counters of every handle
+        if (cudaMemsetAsync(fsms[i]->d_stats, 0, sizeof(DevStats), lead->stream) != cudaSuccess) {
+            restore();
+            return FSM_ECUDA;
+        }
     std::vector<int> group_of(m, -1);
     std::vector<Params> hp(m);
     int rc = FSM_OK;
@@ -1177,7 +1327,7 @@ extern "C" int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *inpu
         }
         if (lead->opt.ctas_per_sm) occ = std::min<int>(occ, (int)lead->opt.ctas_per_sm);
         const uint64_t ntickets = (uint64_t)gp.ntiles * M;
-        const uint32_t grid = (uint32_t)std::min<uint64_t>(ntickets, (uint64_t)occ * lead->num_sms);
+        const uint32_t grid = (uint32_t)std::min<uint64_t>(ntickets, (uint64_t)occ * grid_sms(lead));
         gp.ticket = lead->d_ticket;
         gp.ticket_base = lead->ticket_base;
         fn<<<grid, T, smem, lead->stream>>>(gp, lead->d_multi + base, M);

@@ -185,18 +185,6 @@ inline std::vector<uint8_t> image_packed(const ByteDFA &d, bool wide)
     return img;
 }
 
-// H8 (byte mode, N <= 8): per symbol two u32 half rows; field = (next & 3) | count << 4 | (next >> 2) << 7.
-inline std::vector<uint8_t> image_h8(const ByteDFA &d)
-{
-    std::vector<uint8_t> img(256 * 8, 0);
-    for (uint32_t c = 0; c < 256; c++)
-        for (uint32_t s = 0; s < d.n; s++) {
-            const uint32_t nx = d.next[(size_t)s * 256 + c], k = d.inc[(size_t)s * 256 + c];
-            img[c * 8 + (s >> 2) * 4 + (s & 3)] = (uint8_t)((nx & 3) | (k << 4) | ((nx >> 2) << 7));
-        }
-    return img;
-}
-
 // N8 (byte mode, N <= 8): per symbol one u32 row of 4-bit fields, field s = next | count << 3.
 inline std::vector<uint8_t> image_n8(const ByteDFA &d)
 {

@@ -30,7 +30,7 @@ __global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb
     const uint64_t nch = p.len == 0 ? 1 : (p.len + p.chunk - 1) / p.chunk;
     const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
     for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nch; g += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t b = g * p.chunk, e = min(b + p.chunk, p.len);
+        const uint64_t b = max(g * p.chunk, (uint64_t)p.head), e = min((g + 1) * p.chunk, p.len);
         uint32_t S[K], Xc[kExt];
         speculate<K>(tb, p, b, g == 0, false, start_state, S, Xc);
         uint32_t cur[K], acc[K], accf[K];
@@ -81,7 +81,7 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
     __syncthreads();
     uint32_t x = p.start_dev ? p.start_dev->final_state : p.start_state;
     unsigned long long total = p.start_dev ? p.start_dev->count : 0ull;
-    unsigned long long reexec = 0, rebytes = 0;
+    unsigned long long reexec = 0, rebytes = 0, maxchain = 0, chain = 0;
     for (uint64_t batch = 0; batch < nbatch; batch++) {
         const int buf = batch & 1;
         if (threadIdx.x != 0) {
@@ -98,10 +98,11 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
                 if (hit >= 0) {
                     total += bC[buf * T * K + i * K + hit];
                     x = bE[buf * T * K + i * K + hit];
+                    chain = 0;
                     continue;
                 }
                 // re-execute the chunk from the true state (Fig. 4a), early exit on convergence
-                const uint64_t b = (g0 + i) * p.chunk, e = min(b + p.chunk, p.len);
+                const uint64_t b = max((g0 + i) * p.chunk, (uint64_t)p.head), e = min((g0 + i + 1) * p.chunk, p.len);
                 uint32_t y[K], cy[K];
                 bool pres[K];
 #pragma unroll
@@ -128,6 +129,8 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
                 }
                 reexec++;
                 rebytes += pos - b;
+                chain++;  // consecutive re-executed chunks (reset by a speculated hit)
+                maxchain = chain > maxchain ? chain : maxchain;
                 if (conv >= 0) {
                     total += (unsigned long long)cx - cyc + bC[buf * T * K + i * K + conv];
                     x = bE[buf * T * K + i * K + conv];
@@ -154,8 +157,9 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
             p.user_out[2] = (uint32_t)total;
             p.user_out[3] = (uint32_t)(total >> 32);
         }
-        atomicAdd(&p.stats->reexec_chunks, reexec);
-        atomicAdd(&p.stats->reexec_bytes, rebytes);
+        atomicAdd(&p.stats->reexec_true, reexec);  // the walker follows the true path only
+        atomicAdd(&p.stats->reexec_true_bytes, rebytes);
+        atomicMax(&p.stats->max_miss_chain, maxchain);
     }
 }
 

@@ -29,11 +29,11 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
     const uint32_t start_state = p.start_dev ? p.start_dev->final_state : p.start_state;
     for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nch; g += (uint64_t)gridDim.x * blockDim.x) {
         uint16_t *out = spec + g * stride;
-        const uint64_t b = g * p.chunk;
+        const uint64_t b = max(g * p.chunk, (uint64_t)p.head);
         uint32_t written = 0;
         if (g == 0 && !p.keyed) {
             out[written++] = (uint16_t)start_state;
-        } else if (b >= Lw + 1 && p.aligned) {
+        } else if (b >= Lw + 1 + p.head && p.aligned) {
             const uint32_t c0 = __ldg(p.in + b - Lw - 1);
             const uint32_t ni = __ldg(p.nimg + c0);
             // the image chains run in the table variant's own hot-loop form (its step(), on groups of
@@ -86,10 +86,11 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
                     if (y[i] == bs) mult[i] = 0;
                 out[written] = (uint16_t)bs;
             }
-        } else if (!p.keyed && b > 0) {
-            // the window would reach the start of a known-start run: exact state
+        } else if (!p.keyed && b <= Lw + p.head) {
+            // the window would reach the start of a known-start run: the exact state (at most Lw
+            // bytes from the start)
             uint32_t st = start_state, dummy = 0;
-            for (uint64_t t = 0; t < b; t++) st = tb.apply(tb.row(__ldg(p.in + t)), st, dummy);
+            for (uint64_t t = p.head; t < b; t++) st = tb.apply(tb.row(__ldg(p.in + t)), st, dummy);
             out[written++] = (uint16_t)st;
         } else {
             const uint32_t c = g == 0 ? p.halo_byte : (uint32_t)__ldg(p.in + b - 1);

@@ -27,7 +27,7 @@
 
 namespace speck {
 
-enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, VAR_H8 = 4, VAR_HS = 5, VAR_CL = 6, VAR_N8 = 7, VAR_R16 = 8 };
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, /* 4: retired (H8) */ VAR_HS = 5, VAR_CL = 6, VAR_N8 = 7, VAR_R16 = 8 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
 // in lockstep over the chunk's first kExtWindow bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
@@ -39,10 +39,7 @@ constexpr uint32_t kExtNone = 0xFFFFu;
 // caps them for large K.
 // (K = 2, 3 at 768 threads get 85 registers: the multi-chain prologue spills at 64; measured
 // +6 % over 1024 threads for (8, 2, k=2).)
-#ifndef FSM_T1
-#define FSM_T1 1024
-#endif
-__host__ __device__ constexpr int max_threads(int K) { return K == 1 ? FSM_T1 : K <= 3 ? 768 : K <= 6 ? 512 : 256; }
+__host__ __device__ constexpr int max_threads(int K) { return K == 1 ? 1024 : K <= 3 ? 768 : K <= 6 ? 512 : 256; }
 __host__ __device__ constexpr int min_blocks(int) { return 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
 
@@ -71,37 +68,8 @@ __device__ __forceinline__ Bytes32 ldg256(const uint8_t *p)
                  : "l"(p));
     return r;
 }
-// Same load with an L2 fetch-size hint: the L2 pulls 256 B from DRAM, so the lane's next seven
-// 32-byte blocks arrive from L2 instead of HBM (deeper effective prefetch without registers).
-__device__ __forceinline__ Bytes32 ldg256_l2pf(const uint8_t *p)
-{
-    Bytes32 r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-                 : "=r"(r.w[0]), "=r"(r.w[1]), "=r"(r.w[2]), "=r"(r.w[3]), "=r"(r.w[4]), "=r"(r.w[5]),
-                   "=r"(r.w[6]), "=r"(r.w[7])
-                 : "l"(p));
-    return r;
-}
-__device__ __forceinline__ void prefetch_l2(const uint8_t *p)
-{
-    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
-}
-#ifndef FSM_LOADMODE
-#define FSM_LOADMODE 0
-#endif
-// streaming load of block i of the chunk (FSM_LOADMODE 0: plain, 1: L2::256B hint, 2: plain +
-// explicit L2 prefetch 8 blocks ahead)
-__device__ __forceinline__ Bytes32 ldg_block(const uint8_t *p, uint64_t i, uint64_t nblk)
-{
-#if FSM_LOADMODE == 1
-    return ldg256_l2pf(p + 32 * i);
-#elif FSM_LOADMODE == 2
-    if (i + 8 < nblk) prefetch_l2(p + 32 * (i + 8));
-    return ldg256(p + 32 * i);
-#else
-    return ldg256(p + 32 * i);
-#endif
-}
+// streaming load of 32-byte block i of a chunk
+__device__ __forceinline__ Bytes32 ldg_block(const uint8_t *p, uint64_t i) { return ldg256(p + 32 * i); }
 __device__ __forceinline__ uint4 ldg128(const uint8_t *p)
 {
     return __ldg(reinterpret_cast<const uint4 *>(p));
@@ -160,7 +128,7 @@ __device__ __forceinline__ uint32_t dp4a_u(uint32_t a, uint32_t b, uint32_t c)
 }
 constexpr uint32_t kPackedBase = 0x10000u;  // shared-window address of the packed tables
 constexpr uint32_t kSmemWindowBase = 1024u;  // dynamic shared memory starts here (measured: tools/smem_probe)
-__host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1 || var == 4 || var == 7; }
+__host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1 || var == 7; }
 // CL: the entry table sits at the start of dynamic smem (shared address 0x400 up to < 0x20000) and
 // the 32 KiB lane-replicated class map at the fixed shared address 0x20000, so a class-map address
 // is (byte << 7) | lane * 4 | 0x20000 -- disjoint bit fields, one LOP3 after the byte's shift.
@@ -287,79 +255,21 @@ struct TablePacked {
     }
 };
 
-// H8: N <= 8, byte mode.  Each row is split into two 4-state halves (states 0-3, 4-7) stored as
-// two lane-replicated u32 words at 0x10000 + c * 256 + half * 128 + lane * 4.  A chain loads only
-// the half its current state lives in: ONE conflict-free LDS.32 (one wavefront) instead of P8's
-// LDS.64 (two), at the price of putting the load on the dependency chain.  Field byte:
-// bits 0-1 = index in the half (PRMT selector), bit 4 = accept increment, bit 7 = half, so the
-// address of the next load is one LOP3: (cur & 0x80) | (PRMT of the input byte).
-struct TableH8 {
-    uint32_t lanereg;
-    uint32_t c27, c2;
-    __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
-    {
-        lanereg = kPackedBase | ((threadIdx.x & 31) * 4);
-        c27 = kc.k_1e27;
-        c2 = kc.k_2;
-        const uint2 *rows = static_cast<const uint2 *>(g);  // per symbol: {half 0 word, half 1 word}
-        for (uint32_t i = threadIdx.x; i < 256 * 64; i += blockDim.x) {
-            const uint32_t c = i >> 6, h = (i >> 5) & 1, l = i & 31;
-            const uint2 v = __ldg(rows + c);
-            asm volatile("st.shared.u32 [%0], %1;" ::"r"(kPackedBase + c * 256 + h * 128 + l * 4), "r"(h ? v.y : v.x));
-        }
-    }
-    __device__ __forceinline__ uint32_t init(uint32_t st) const { return (st & 3u) | ((st & 4u) << 5); }
-    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return (cur & 3u) | ((cur >> 5) & 4u); }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
-    template <int K>
-    __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
-                                         uint32_t (&accf)[K]) const
-    {
-        const uint32_t a = prmt(w, lanereg, 0x7604u | (uint32_t(j) << 4));
-#pragma unroll
-        for (int s = 0; s < K; s++) {
-            const uint32_t r = lds_u32(a | (cur[s] & 0x80u));   // LOP3 + LDS.32 (half of the row)
-            cur[s] = prmt(r, r, cur[s]);                         // select the field
-            accf[s] = mad_hi(cur[s] * c27, c2, accf[s]);         // + bit 4, on the FMA pipe
-        }
-    }
-    using Row = uint2;
-    __device__ __forceinline__ Row row(uint32_t c) const
-    {
-        const uint32_t a = lanereg + (c << 8);
-        return make_uint2(lds_u32(a), lds_u32(a + 128));
-    }
-    __device__ __forceinline__ uint32_t apply(Row r, uint32_t st, uint32_t &cnt) const
-    {
-        const uint32_t w = (st & 4u) ? r.y : r.x;
-        const uint32_t f = prmt(w, w, st & 3u) & 0xFFu;
-        cnt += (f >> 4) & 1u;
-        return (f & 3u) | ((f >> 5) & 4u);
-    }
-};
-
 // N8: N <= 8, byte mode.  The transition function of symbol c is ONE 32-bit row of eight 4-bit
 // fields, field s = next | count << 3, lane-replicated at 0x10000 + c * 256 + lane * 4 (P4's layout,
 // so the address is one PRMT of the input word and the load is one conflict-free LDS.32 = one
 // wavefront per byte per warp, half of P8's LDS.64).  A chain carries the shift amount 4 * state:
 // t = funnel-shift-right(row, cur) in wrap mode (only cur & 31 is used), and the next shift amount
 // is t * 4, whose bits 2..4 are t's next-state bits -- the garbage above bit 4 is ignored by the
-// next wrap-mode shift.  Chain step: SHF.R.W (ALU) + IMAD (FMA); count bit = bit 3 of t, added on
-// the ALU (LOP3 + half an IADD3) and FMA (IMAD + IMAD.HI) pipes on alternate steps.
+// next wrap-mode shift.  Chain step: SHF.R.W (ALU) + IMAD (FMA); the count bit = bit 3 of t is
+// summed four bytes at a time (step4).
 struct TableN8 {
     uint32_t lanereg;
-    uint32_t c4, c28, c2, c24, c16x, c8x, c256, c26;
+    uint32_t c4;
     __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
     {
         lanereg = kPackedBase | ((threadIdx.x & 31) * 4);
         c4 = kc.k_4;
-        c28 = kc.k_1e28;
-        c2 = kc.k_2;
-        c24 = kc.k_1e24;          // 1 << 24
-        c16x = kc.k_16 << 12;     // 1 << 16
-        c8x = kc.k_16 << 4;       // 1 << 8
-        c256 = kc.k_512 >> 1;     // 256
-        c26 = kc.k_1e24 << 2;     // 1 << 26
         const uint32_t *rows = static_cast<const uint32_t *>(g);
         for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
             const uint32_t v = __ldg(rows + (i >> 5));
@@ -374,12 +284,11 @@ struct TableN8 {
     }
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st * 4u; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return (cur >> 2) & 7u; }
-    // Without step4: acc = 8 * (ALU-counted steps), accf = FMA-counted steps.  With step4: accf
-    // counts in units of 32 (DP4A / LOP3 of bit 5 of v, and the byte tail), acc in units of 1 (the
-    // hybrid FSM_N8_BATCH == 2 FMA part).
+    // accf counts in units of 32 (the DP4A of bit 5 of v in step4, and the byte tails in step); acc
+    // is unused.
     __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const
     {
-        return kStep4 ? acc + (accf >> 5) : (acc >> 3) + accf;
+        return acc + (accf >> 5);
     }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
@@ -390,37 +299,19 @@ struct TableN8 {
         for (int s = 0; s < K; s++) {
             const uint32_t t = shr_wrap(r, cur[s]);          // field of the current state in bits 0..3
             cur[s] = mad_lo(t, c4, 0u);                      // next shift amount (bits 2..4 valid)
-            if (kStep4) accf[s] += (t & 8u) << 2;                 // byte tails of step4 chunks: units of 32
-            else if (((j + s) & 1) == 0) acc[s] += t & 8u;        // ALU: LOP3 (+ half an IADD3)
-            else accf[s] = mad_hi(t * c28, c2, accf[s]);          // FMA: IMAD, IMAD.HI (bit 3 of t)
+            accf[s] += (t & 8u) << 2;                        // byte tails of step4 chunks: units of 32
         }
     }
-#ifndef FSM_N8_BATCH
-#define FSM_N8_BATCH 1
-#endif
-#ifndef FSM_N8_FMA_ADDR
-#define FSM_N8_FMA_ADDR 0
-#endif
     // Four bytes of word w at once: the four rows are loaded up front, and the count of the four
     // steps is taken in one go -- the next shift amounts v = 4t carry the accept bit in bit 5; their
     // low bytes are gathered by two PRMTs into one word, masked, and summed by one DP4A (acc counts
     // in units of 32).  ALU: 4 address PRMT + 4 SHF + 3 PRMT + 1 LOP3; FMA: 4 IMAD + 1 DP4A.
-    static constexpr bool kStep4 = FSM_N8_BATCH != 0;
     template <int K>
     __device__ __forceinline__ void step4(uint32_t w, uint32_t (&cur)[K], uint32_t (&acc)[K], uint32_t (&accf2)[K]) const
     {
         uint32_t r[4];
-#if FSM_N8_FMA_ADDR
-        // bytes 0 and 3 addressed on the FMA pipe (the ALU pipe is the binding one):
-        //   byte 0: x = w << 24 (IMAD), addr = (x >> 16) + lanereg (IMAD.HI);  byte 3: (w >> 24) * 256 + lanereg
-        r[0] = lds_u32(mad_hi(mad_lo(w, c24, 0u), c16x, lanereg));
-        r[1] = lds_u32(prmt(w, lanereg, 0x7614u));
-        r[2] = lds_u32(prmt(w, lanereg, 0x7624u));
-        r[3] = lds_u32(mad_lo(mad_hi(w, c8x, 0u), c256, lanereg));
-#else
 #pragma unroll
         for (int j = 0; j < 4; j++) r[j] = lds_u32(prmt(w, lanereg, 0x7604u | (uint32_t(j) << 4)));
-#endif
 #pragma unroll
         for (int s = 0; s < K; s++) {
             uint32_t v[4];
@@ -431,16 +322,8 @@ struct TableN8 {
                 c = v[j];
             }
             cur[s] = c;
-#if FSM_N8_BATCH == 2
-            // hybrid: steps 0, 1 counted on the FMA pipe (IMAD + IMAD.HI of bit 5 of v), steps 2, 3 on
-            // the ALU pipe (two LOP3 + one IADD3), in units of 32 -- moves work off the busy ALU pipe
-            accf2[s] = mad_hi(mad_lo(v[0], c26, 0u), c2, accf2[s]);
-            accf2[s] = mad_hi(mad_lo(v[1], c26, 0u), c2, accf2[s]);
-            acc[s] += (v[2] & 32u) + (v[3] & 32u);
-#else
             const uint32_t lo = prmt(v[0], v[1], 0x0040u), hi = prmt(v[2], v[3], 0x0040u);
             acc[s] = dp4a_u(prmt(lo, hi, 0x5410u) & 0x20202020u, 0x01010101u, acc[s]);
-#endif
         }
     }
     using Row = uint32_t;
@@ -661,6 +544,15 @@ struct TableR16 {
     {
         return (acc >> 4) + (cur >> 4) + accf;
     }
+    // Move the pending (one-step-late) count of the last entry into the accumulator.  Needed before
+    // the convergence collapse replaces every slot's chain by slot 0's: in bit mode the pending count
+    // (F-visits of the last widened byte) depends on the slot's own source state, not only on the
+    // common destination.
+    __device__ __forceinline__ void settle(uint32_t &cur, uint32_t &acc) const
+    {
+        acc += cur & ~0xFu;
+        cur &= 0xFu;
+    }
     // symbol part of the address of byte j of w
     __device__ __forceinline__ uint32_t sym(uint32_t w, int j) const
     {
@@ -694,7 +586,6 @@ template <> struct TableFor<VAR_P4> { using type = TablePacked<VAR_P4>; };
 template <> struct TableFor<VAR_P8> { using type = TablePacked<VAR_P8>; };
 template <> struct TableFor<VAR_B> { using type = TableB; };
 template <> struct TableFor<VAR_G> { using type = TableG; };
-template <> struct TableFor<VAR_H8> { using type = TableH8; };
 template <> struct TableFor<VAR_HS> { using type = TableHS; };
 template <> struct TableFor<VAR_CL> { using type = TableCL; };
 template <> struct TableFor<VAR_N8> { using type = TableN8; };
@@ -702,7 +593,12 @@ template <> struct TableFor<VAR_R16> { using type = TableR16; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <class TB> struct TableHasStep4 { static constexpr bool value = false; };
-template <> struct TableHasStep4<TableN8> { static constexpr bool value = TableN8::kStep4; };
+// Tables whose chain value carries a count not yet added to the accumulator (R16) settle it before
+// the convergence collapse.  P4 also lags its count, but only in byte mode, where the count of an
+// entry is that of its destination state and so equal in every converged slot.
+template <class TB> struct TableHasSettle { static constexpr bool value = false; };
+template <> struct TableHasSettle<TableR16> { static constexpr bool value = true; };
+template <> struct TableHasStep4<TableN8> { static constexpr bool value = true; };
 
 template <int K, class TB>
 __device__ __forceinline__ void process32(const TB &tb, const Bytes32 &x, uint32_t (&cur)[K], uint32_t (&acc)[K],
@@ -749,41 +645,14 @@ __device__ __forceinline__ bool chains_converged(const TB &tb, const uint32_t (&
 // Blocks [i, nblk) of 32 bytes with a 3-buffer rotation (2 blocks in flight, no register moves).
 // On entry x0 = block i, x1 = block i+1.  With CHECK, returns true as soon as the warp votes
 // that all chains coincide; x0/x1 then hold blocks i, i+1 for the continuation.
-#ifndef FSM_NBUF
-#define FSM_NBUF 3
-#endif
 template <int KK, bool CHECK, class TB>
 __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint64_t &i, uint64_t nblk, Bytes32 &x0,
                                            Bytes32 &x1, uint32_t (&cur)[KK], uint32_t (&acc)[KK],
                                            uint32_t (&accf)[KK])
 {
-#if FSM_NBUF == 2
-    // two buffers: block i+2 is requested after block i is consumed (16 registers of input in
-    // flight instead of 24; the freed registers let the table-row loads run ahead of their use)
-    while (i < nblk) {
-        process32<KK>(tb, x0, cur, acc, accf);
-        ++i;
-        if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
-            x0 = x1;
-            if (i + 1 < nblk) x1 = ldg_block(p, i + 1, nblk);
-            return true;
-        }
-        if (i >= nblk) break;
-        if (i + 1 < nblk) x0 = ldg_block(p, i + 1, nblk);
-        process32<KK>(tb, x1, cur, acc, accf);
-        ++i;
-        if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
-            if (i + 1 < nblk) x1 = ldg_block(p, i + 1, nblk);  // x0 already holds block i
-            return true;
-        }
-        if (i >= nblk) break;
-        if (i + 1 < nblk) x1 = ldg_block(p, i + 1, nblk);
-    }
-    return false;
-#else
     Bytes32 x2;
     while (i < nblk) {
-        if (i + 2 < nblk) x2 = ldg_block(p, i + 2, nblk);
+        if (i + 2 < nblk) x2 = ldg_block(p, i + 2);
         process32<KK>(tb, x0, cur, acc, accf);
         ++i;
         if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
@@ -792,7 +661,7 @@ __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint6
             return true;
         }
         if (i >= nblk) break;
-        if (i + 2 < nblk) x0 = ldg_block(p, i + 2, nblk);
+        if (i + 2 < nblk) x0 = ldg_block(p, i + 2);
         process32<KK>(tb, x1, cur, acc, accf);
         ++i;
         if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
@@ -801,7 +670,7 @@ __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint6
             return true;
         }
         if (i >= nblk) break;
-        if (i + 2 < nblk) x1 = ldg_block(p, i + 2, nblk);
+        if (i + 2 < nblk) x1 = ldg_block(p, i + 2);
         process32<KK>(tb, x2, cur, acc, accf);
         ++i;
         if (CHECK && __all_sync(__activemask(), chains_converged<KK>(tb, cur))) {
@@ -810,7 +679,6 @@ __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint6
         }
     }
     return false;
-#endif
 }
 
 // Alg. 3 over bytes [b, e) of the input: 32-byte blocks (one full sector per lane per
@@ -825,6 +693,13 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
                                             bool aligned, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                             uint32_t (&accf)[K], uint32_t *stash = nullptr)
 {
+    if (aligned && (b & 31)) {
+        // the peeled head of an unaligned input (chunk 0 starts at in + head): bytes up to the first
+        // 32-byte boundary one at a time, then full sectors
+        const uint64_t stop = min(e, (b + 31) & ~(uint64_t)31);
+        for (; b < stop; b++) tb.template step<K>(__ldg(in + b), 0, cur, acc, accf);
+        stash = nullptr;
+    }
     const uint8_t *p = in + b;
     const uint64_t n = e - b;
     const uint64_t nblk = aligned ? (n >> 5) : 0;
@@ -832,8 +707,8 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
     bool single = false;
     Bytes32 x0, x1;
     if (nblk) {
-        x0 = ldg_block(p, 0, nblk);
-        if (nblk > 1) x1 = ldg_block(p, 1, nblk);
+        x0 = ldg_block(p, 0);
+        if (nblk > 1) x1 = ldg_block(p, 1);
         if (stash) {
             reinterpret_cast<uint4 *>(stash)[0] = make_uint4(x0.w[0], x0.w[1], x0.w[2], x0.w[3]);
             reinterpret_cast<uint4 *>(stash)[1] = make_uint4(x0.w[4], x0.w[5], x0.w[6], x0.w[7]);
@@ -842,6 +717,10 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
     }
     if constexpr (K > 1) {
         if (single) {
+            if constexpr (TableHasSettle<TB>::value) {
+#pragma unroll
+                for (int s = 0; s < K; s++) tb.settle(cur[s], acc[s]);
+            }
             uint32_t c1[1] = {cur[0]}, a1[1] = {0u}, f1[1] = {0u};
             run_blocks<1, false>(tb, p, i, nblk, x0, x1, c1, a1, f1);
             for (uint64_t t = nblk << 5; t < n; t++) tb.template step<1>(__ldg(p + t), 0, c1, a1, f1);
@@ -878,7 +757,7 @@ __device__ __forceinline__ void speculate(const TB &tb, const Params &p, uint64_
 #pragma unroll
     for (int q = 0; q < kExt; q++) X[q] = NOSTATE;
     if (empty) return;
-    if (first_chunk && !p.keyed) {
+    if (first_chunk && !p.keyed && !p.spec_all) {
         S[0] = start_state;
         return;
     }
@@ -958,16 +837,30 @@ __device__ __forceinline__ void compose(uint32_t (&eob)[K], uint32_t (&cnt)[K], 
     }
 }
 
-// Warp-level suffix scan (Kogge-Stone over shuffles): afterwards lane i holds the mapping of
-// elements [i, 32) keyed on its own start set.  first0 = chunk index of lane 0's element, step =
-// chunk distance between lanes.
+// Test hook (fsm_debug_get_merge): the lane's mapping after scan level `level` (0 = the chunk's own).
 template <int K>
-__device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eob)[K], uint32_t (&cnt)[K], bool &ident,
-                                                 uint32_t first0, uint32_t step, const uint32_t *ext = nullptr)
+__device__ __forceinline__ void dbg_record(uint4 *dbg, int level, const uint32_t (&S)[K], const uint32_t (&eob)[K],
+                                           const uint32_t (&cnt)[K], bool ident)
 {
     const int lane = threadIdx.x & 31;
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
+    for (int s = 0; s < K; s++) dbg[(level * 32 + lane) * KMAX + s] = make_uint4(S[s], eob[s], cnt[s], ident ? 1u : 0u);
+}
+
+// Warp-level suffix scan (Kogge-Stone over shuffles): afterwards lane i holds the mapping of
+// elements [i, 32) keyed on its own start set.  first0 = chunk index of lane 0's element, step =
+// chunk distance between lanes.  Level d composes lane i with lane i + d, so lane 0 after d = 1 is
+// M_0 x M_1, lane 2 is M_2 x M_3, and lane 0 after d = 2 is (M_0 x M_1) x (M_2 x M_3): the merge tree
+// of Fig. 4b.  dbg (test hook, normally null) records every level.
+template <int K>
+__device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eob)[K], uint32_t (&cnt)[K], bool &ident,
+                                                 uint32_t first0, uint32_t step, const uint32_t *ext = nullptr,
+                                                 uint4 *dbg = nullptr)
+{
+    const int lane = threadIdx.x & 31;
+    if (dbg) dbg_record<K>(dbg, 0, S, eob, cnt, ident);
+#pragma unroll
+    for (int d = 1, level = 1; d < 32; d <<= 1, level++) {
         uint32_t Sr[K], er[K], cr[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
@@ -977,6 +870,7 @@ __device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eo
         }
         const bool ir = __shfl_down_sync(0xFFFFFFFFu, (int)ident, d) != 0;
         if (lane + d < 32 && !ir && !ident) compose<K>(eob, cnt, Sr, er, cr, first0 + (lane + d) * step, ext);
+        if (dbg) dbg_record<K>(dbg, level, S, eob, cnt, ident);
     }
 }
 
@@ -1037,7 +931,7 @@ __host__ __device__ constexpr bool split_kernel(int var, int K)
 {
     return FSM_SPLIT == 1 ? true
          : FSM_SPLIT == 0 ? false
-         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 4 || var == 2 || var == 7 || var == 8) /* P4 P8 H8 B N8 R16 */ && K >= 2));
+         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 2 || var == 7 || var == 8) /* P4 P8 B N8 R16 */ && K >= 2));
 }
 
 // Per-tile context used by re-execution and the epilogue.
@@ -1045,6 +939,7 @@ struct TileCtx {
     const uint8_t *in;
     uint64_t len;
     uint64_t tile_base;
+    uint32_t head;      // chunk 0 of the run starts at in + head (peeled unaligned input)
     uint32_t chunk;
     uint32_t nch;       // non-empty chunks in this tile (>= 1)
     bool aligned;
@@ -1075,15 +970,20 @@ __device__ __forceinline__ int ext_lookup(const uint32_t *ext, uint32_t c, uint3
 // ("re-execute the next chunk with states[s]"); the moment the re-executed state equals a
 // speculated chain's state both runs coincide for the rest of the chunk, so the result is exact:
 // (that chain's path, n + cnt_x(p) - cnt_l(p) + its count).  Otherwise continue at chunk c+1.
+// The work done is tallied in rc (chunks, bytes, longest run of consecutive re-executed chunks,
+// eager-entry completions); the caller attributes it to the true or a candidate path.
 template <int K, class TB>
 __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c, uint32_t n, uint32_t &out_st,
-                        uint32_t &out_n)
+                        uint32_t &out_n, ReCount &rc)
 {
+    uint32_t chain = 0, last_c = 0xFFFFFFFFu;
     for (;;) {
         {   // eager completion already ran this state into one of the chunk's chains
             int32_t dl;
             const int l = ext_lookup(t.ext, c, st, dl);
             if (l >= 0) {
+                rc.eager++;
+                if (c == 0 && rc.chunks == 0) rc.join0 = (uint32_t)l;
                 n += (uint32_t)dl + t.Qc[c * K + l];
                 const uint32_t x = t.Qe[c * K + l];
                 if ((x >> 16) == COMPLETE) {
@@ -1096,8 +996,8 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
                 continue;
             }
         }
-        const uint64_t b = t.tile_base + (uint64_t)c * t.chunk;
-        const uint64_t e = min(b + t.chunk, t.len);
+        const uint64_t b = max(t.tile_base + (uint64_t)c * t.chunk, (uint64_t)t.head);
+        const uint64_t e = min(t.tile_base + (uint64_t)(c + 1) * t.chunk, t.len);
         uint32_t y[K], cy[K];
         bool pres[K];
 #pragma unroll
@@ -1122,7 +1022,7 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
                     cyc = cy[l];
                 }
         };
-        if (t.stash && t.aligned && e - b >= 32) {
+        if (t.stash && t.aligned && (b & 31) == 0 && e - b >= 32) {
             // the chunk's first 32 bytes were stashed in smem by its owner during the local phase:
             // the usual early exit never touches global memory
 #pragma unroll 1
@@ -1132,6 +1032,10 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
             }
         }
         if (t.aligned) {
+            while (conv < 0 && (pos & 15) && pos < e) {
+                one(__ldg(t.in + pos));
+                pos++;
+            }
             while (conv < 0 && pos + 16 <= e) {
                 const uint4 v = ldg128(t.in + pos);
                 uint32_t used = 0;
@@ -1148,10 +1052,14 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
             one(__ldg(t.in + pos));
             pos++;
         }
-        atomicAdd(&t.stats->reexec_chunks, 1ull);
-        atomicAdd(&t.stats->reexec_bytes, (unsigned long long)(pos - b));
+        chain = c == last_c + 1 ? chain + 1 : 1;
+        last_c = c;
+        rc.chunks++;
+        rc.bytes += (uint32_t)(pos - b);
+        rc.chain = max(rc.chain, chain);
         uint32_t x;
         if (conv >= 0) {
+            if (c == 0 && rc.chunks == 1) rc.join0 = (uint32_t)conv;
             n += cx - cyc + t.Qc[c * K + conv];
             x = t.Qe[c * K + conv];
         } else {
@@ -1179,9 +1087,27 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
     }
 }
 
+__device__ __forceinline__ void add_stats(DevStats *S, const ReCount &rc, bool true_path)
+{
+    if (!rc.chunks && !rc.eager) return;
+    if (true_path) {
+        if (rc.chunks) {
+            atomicAdd(&S->reexec_true, (unsigned long long)rc.chunks);
+            atomicAdd(&S->reexec_true_bytes, (unsigned long long)rc.bytes);
+            atomicMax(&S->max_miss_chain, (unsigned long long)rc.chain);
+        }
+        if (rc.eager) atomicAdd(&S->eager_resolved, (unsigned long long)rc.eager);
+    } else if (rc.chunks) {
+        atomicAdd(&S->reexec_cand, (unsigned long long)rc.chunks);
+        atomicAdd(&S->reexec_cand_bytes, (unsigned long long)rc.bytes);
+    }
+}
+
 // a7-a9 for one tile, run by one full warp once the tile's suffix mappings Qe/Qc (keyed on the
 // chunks' speculated starts Sj) are in shared memory: pre-resolution of the tile aggregate's broken
-// slots (R5), publication of A, decoupled look-back, own inclusive prefix P, and the result.
+// slots (R5, the top p.preresolve tile-start candidates), publication of A, decoupled look-back,
+// own inclusive prefix P (resolving the true path's broken slot if it was left unresolved), and the
+// result.
 template <int K, class TB>
 __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uint32_t tile, uint64_t tile_base,
                                               uint32_t nch_max, uint32_t *Qe, uint32_t *Qc, const uint16_t *Sj,
@@ -1193,6 +1119,7 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
     t.in = p.in;
     t.len = p.len;
     t.tile_base = tile_base;
+    t.head = p.head;
     t.chunk = p.chunk;
     {
         const uint64_t rem = p.len > tile_base ? p.len - tile_base : 0;
@@ -1207,24 +1134,30 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
     t.ext = Ext;
     t.stats = p.stats;
 
-    // a8 (tile candidates): resolve the broken slots of the tile aggregate Q_0 so that the
-    // published aggregate is complete on every speculated tile start.
-    if (lane < K) {
-        const uint32_t x = Qe[lane];
-        if ((x >> 16) < ABSENT) {
+    // a8 (tile candidates, R5): resolve the broken slots of the tile aggregate Q_0 for the top
+    // p.preresolve speculated tile starts, so that a successor's look-back can pass through them
+    // without waiting for this tile's P.  The other slots are published broken (lazy): they are
+    // resolved only if the true path turns out to enter this tile in them.
+    ReCount rc5{0, 0, 0, 0, 0xFFFFu};
+    uint32_t qe = lane < K ? Qe[lane] : 0u, qc = lane < K ? Qc[lane] : 0u;  // own-prefix source
+    if (lane < K && (uint32_t)lane < p.preresolve) {
+        if ((qe >> 16) < ABSENT) {
             uint32_t st, n;
-            resolve<K>(tb, t, x & 0xFFFFu, x >> 16, Qc[lane], st, n);
-            Qe[lane] = st | (COMPLETE << 16);
-            Qc[lane] = n;
+            resolve<K>(tb, t, qe & 0xFFFFu, qe >> 16, qc, st, n, rc5);
+            qe = st | (COMPLETE << 16);
+            qc = n;
+            Qe[lane] = qe;  // a later tile-boundary re-execution that joins this slot reuses it
+            Qc[lane] = qc;
         }
     }
     __syncwarp();
 
-    // a7: publish the aggregate A_b (slot = {start, end, count})
+    // a7: publish the aggregate A_b (slot = {start, end, count, broken})
     TileDesc *D = p.desc + tile;
     if (lane < K) {
         const uint32_t sv = Sj[lane];
-        D->aslot[lane] = make_uint4(sv == 0xFFFFu ? NOSTATE : sv, Qe[lane] & 0xFFFFu, Qc[lane], 0u);
+        const bool broken = (qe >> 16) != COMPLETE;
+        D->aslot[lane] = make_uint4(sv == 0xFFFFu ? NOSTATE : sv, qe & 0xFFFFu, qc, broken ? 1u : 0u);
     }
     __threadfence();
     __syncwarp();
@@ -1289,7 +1222,8 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
     // (2) apply the aggregates A_{m+1} .. A_{b-1}, 32 per step: every lane loads one tile's
     // aggregate in parallel, a warp suffix scan composes the 32 mappings (the same operator as
     // the chunk merge), and the composed window is applied to E.  A slot that breaks inside the
-    // window hit a tile-boundary miss there: take that tile's P and continue after it.
+    // window (a tile-boundary miss, or a slot a tile published unresolved) is taken from that
+    // tile's P, and the walk continues after it.
     for (int64_t nx = m + 1; nx < (int64_t)tile;) {
         const int64_t tt = nx + lane;
         uint32_t S2[K], e2[K], c2[K];
@@ -1301,7 +1235,7 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
             for (int l = 0; l < K; l++) {
                 const uint4 v = __ldcg(&Dt->aslot[l]);
                 S2[l] = v.x;
-                e2[l] = v.x == NOSTATE ? (ABSENT << 16) : (v.y | (COMPLETE << 16));
+                e2[l] = v.x == NOSTATE ? (ABSENT << 16) : (v.y | ((v.w ? (uint32_t)lane : COMPLETE) << 16));
                 c2[l] = v.z;
             }
         } else {
@@ -1335,31 +1269,38 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
         }
         const int mb = __reduce_min_sync(0xFFFFFFFFu, brk);
         if (mb < 32) {
-            load_P(nx + mb);  // E := P of the tile where a slot broke (it resolves its own miss)
+            load_P(nx + mb);  // E := P of the tile where a slot broke (it resolves its own true path)
             nx = nx + mb + 1;
         } else {
             nx += 32;
         }
     }
 
-    // own inclusive prefix P_b = E then A_b; a tile-boundary miss resolves through chunk 0.
+    // own inclusive prefix P_b = E then A_b.  A tile-boundary miss (E's state is no speculated tile
+    // start) resolves through chunk 0; a hit on a slot left unresolved resolves from its break.
     uint32_t Ps = 0;
     unsigned long long Pc = 0;
+    ReCount rct{0, 0, 0, 0, 0xFFFFu};
+    // the slot values live in lanes 0..K-1: fetch the hit slot's (qe, qc) with a full-warp shuffle
+    int hit = -1;
     if (Ev) {
-        bool hit = false;
 #pragma unroll
         for (int l = 0; l < K; l++)
-            if (!hit && Sj[l] == Es) {
-                Ps = Qe[l] & 0xFFFFu;
-                Pc = Ec + Qc[l];
-                hit = true;
-            }
-        if (!hit) {
+            if (hit < 0 && Sj[l] == Es) hit = l;
+    }
+    const uint32_t hq = __shfl_sync(0xFFFFFFFFu, qe, hit < 0 ? 0 : hit);
+    const uint32_t hc = __shfl_sync(0xFFFFFFFFu, qc, hit < 0 ? 0 : hit);
+    if (Ev) {
+        if (hit >= 0 && (hq >> 16) == COMPLETE) {
+            Ps = hq & 0xFFFFu;
+            Pc = Ec + hc;
+        } else {
             uint32_t st, n;
-            resolve<K>(tb, t, Es, 0, 0, st, n);
+            if (hit >= 0) resolve<K>(tb, t, hq & 0xFFFFu, hq >> 16, hc, st, n, rct);  // lazy R5 slot
+            else resolve<K>(tb, t, Es, 0, 0, st, n, rct);                               // tile-boundary miss
             Ps = st;
             Pc = Ec + n;
-            atomicAdd(&p.stats->boundary_misses, 1ull);
+            if (hit < 0) atomicAdd(&p.stats->boundary_misses, 1ull);
         }
     }
     const unsigned vmask = __ballot_sync(0xFFFFFFFFu, Ev);
@@ -1371,6 +1312,23 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
     __threadfence();
     __syncwarp();
     if (lane == 0) st_release(&D->flag, ep | ST_P);
+
+    // counters: a pre-resolved slot is on the true path iff some valid prefix slot entered the
+    // tile in its speculated start, or a tile-boundary re-execution joined it in chunk 0 (keyed
+    // mode: every shard slot's path is needed)
+    add_stats(p.stats, rct, true);
+    if (__any_sync(0xFFFFFFFFu, rc5.chunks | rc5.eager)) {
+        const uint32_t mine = lane < K ? (uint32_t)Sj[lane] : 0xFFFFFFFEu;
+        bool needed = false;
+#pragma unroll
+        for (int q = 0; q < KMAX; q++) {
+            const uint32_t eq = __shfl_sync(0xFFFFFFFFu, Es, q);
+            const bool vq = __shfl_sync(0xFFFFFFFFu, (int)Ev, q) != 0;
+            const uint32_t jq = __shfl_sync(0xFFFFFFFFu, rct.join0, q);
+            needed = needed || (vq && (eq == mine || jq == (uint32_t)lane));
+        }
+        add_stats(p.stats, rc5, needed);
+    }
 
     // a9: the last tile writes the result (bit-mode tail applied here)
     if (tile == p.ntiles - 1) {
@@ -1514,10 +1472,11 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
         const uint32_t ksel = p.k;
 
         const uint64_t tile_base = (uint64_t)tile * TW * p.chunk;
-        const uint64_t b = tile_base + (uint64_t)j * p.chunk;
+        const uint64_t b0 = tile_base + (uint64_t)j * p.chunk;
+        const uint64_t b = max(b0, (uint64_t)p.head);  // chunk 0 starts at the peeled head
         const bool first_chunk = tile == 0 && j == 0;
         const bool empty = b >= p.len && !first_chunk;
-        const uint64_t e = b >= p.len ? b : min(b + p.chunk, p.len);
+        const uint64_t e = b >= p.len ? b : min(b0 + p.chunk, p.len);
 
         // ---- a3: speculated start set (+ eager-completion candidates)
         uint32_t S[K], Xc[kExt];
@@ -1550,7 +1509,7 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
             uint32_t ent[kExt];
 #pragma unroll
             for (int q = 0; q < kExt; q++) ent[q] = kExtNone;
-            if (p.eager_window && p.aligned && !empty && e - b >= 32 && Xc[0] != NOSTATE) {
+            if (p.eager_window && p.aligned && (b & 31) == 0 && !empty && e - b >= 32 && Xc[0] != NOSTATE) {
                 uint32_t y[K], cy[K], u[kExt], cu[kExt];
                 bool live[kExt];
 #pragma unroll
@@ -1609,7 +1568,8 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
 #endif
         // ---- a5: warp stage (chunks warp*32 .. warp*32+31)
         __syncwarp();  // the lanes' eager-completion entries are read by the scan
-        warp_suffix_scan<K>(S, eob, cnt, ident, (uint32_t)warp * 32, 1, Ext);
+        warp_suffix_scan<K>(S, eob, cnt, ident, (uint32_t)warp * 32, 1, Ext,
+                            (p.dbg && tile == 0 && warp == 0) ? p.dbg : nullptr);
 
         // ---- a6: block stage
         if (lane == 0) {

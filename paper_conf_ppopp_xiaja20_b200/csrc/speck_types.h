@@ -26,16 +26,32 @@ struct __align__(128) TileDesc {
     uint32_t flag;                 // epoch << 2 | Status
     uint32_t pmask;                // P: valid slots
     uint32_t pad[2];
-    uint4 aslot[KMAX];             // A: {start (NOSTATE = absent), end, count within tile, 0}
+    uint4 aslot[KMAX];             // A: {start (NOSTATE = absent), end, count within tile, broken}
+                                   //    broken != 0: the slot's run breaks inside the tile (lazy R5):
+                                   //    a successor whose path enters it waits for this tile's P
     uint32_t pstate[KMAX];         // P: state after this tile, per shard slot
     unsigned long long pcnt[KMAX]; // P: count up to and including this tile, per shard slot
 };
 
+// Re-execution counters of one run (reset by the host at the start of every API call).  A8: only
+// chunks whose true start was not speculated should be re-executed; re-executions made for a
+// tile-start candidate that turns out not to be on the true path (R5 pre-resolution) are counted
+// apart.  In keyed (shard) mode every valid shard slot's path counts as "true".
 struct DevStats {
-    unsigned long long reexec_chunks;
-    unsigned long long reexec_bytes;
-    unsigned long long boundary_misses;
+    unsigned long long reexec_true;        // chunk re-executions on the true path
+    unsigned long long reexec_true_bytes;  // bytes they consumed (early exit on convergence)
+    unsigned long long reexec_cand;        // re-executions on tile-start candidate paths that were not taken
+    unsigned long long reexec_cand_bytes;
+    unsigned long long boundary_misses;    // tile-boundary misses (true start not a speculated tile start)
+    unsigned long long eager_resolved;     // true-path misses completed from an eager-completion entry
+    unsigned long long max_miss_chain;     // longest run of consecutive re-executed chunks on the true path
     unsigned long long pad;
+};
+
+// Per-slot re-execution tally of one resolve() call.
+struct ReCount {
+    uint32_t chunks, bytes, chain, eager;
+    uint32_t join0;  // slot of chunk 0 that a re-execution starting at chunk 0 joined (0xFFFF = none)
 };
 
 // Result area written by the last tile.
@@ -60,7 +76,10 @@ struct Params {
     uint32_t lookback;             // look-back window in bytes (0/1: the preceding byte only)
     const uint16_t *spec;          // window look-back: ranked candidates per chunk (spec_kernel), or null
     uint32_t spec_stride;          // candidates per chunk in `spec` (k + kExt)
-    uint32_t aligned;              // `in` is 32-byte aligned
+    uint32_t aligned;              // `in` is 32-byte aligned (always, but for tiny debug chunks)
+    uint32_t head;                 // the caller's input starts at in + head (0..31): an unaligned
+                                   // input is run from the aligned address below it, chunk 0 being
+                                   // [head, chunk); every position is relative to `in`, len included
     const void *table;             // variant image in global memory
     uint32_t n_states;             // internal states (incl. sink)
     uint32_t table_bytes;          // bytes of the shared-memory table image (0 for G)
@@ -90,6 +109,9 @@ struct Params {
     uint32_t *user_out;            // optional: the last tile also writes {user state, 0, count lo, hi} here
     uint32_t eager_window;         // NEXT-3 eager completion: bytes of lockstep per chunk (0 = off)
     uint32_t k_4, k_1e28;          // N8 variant: FMA-pipe constants (4, 1 << 28), see k_1e24 above
+    uint32_t preresolve;           // R5: tile-start slots (in rank order) resolved before publishing A
+    uint32_t spec_all;             // test hook: `spec` also overrides chunk 0 of a known-start run
+    uint4 *dbg;                    // test hook: warp-scan levels of tile 0, warp 0 ([6][32][KMAX]), or null
 };
 
 }  // namespace speck

@@ -17,23 +17,26 @@ SO_PATH = os.environ.get("FSMSPEC_SO") or os.path.join(_HERE, "libfsmspec.so")  
 FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 FSM_INPUT_BYTES, FSM_INPUT_BITS_MSB = 0, 1
 FSM_KMAX = 16
-FSM_VARIANT_AUTO, FSM_VARIANT_P4, FSM_VARIANT_P8, FSM_VARIANT_B, FSM_VARIANT_G, FSM_VARIANT_H8 = -1, 0, 1, 2, 3, 4
+FSM_VARIANT_AUTO, FSM_VARIANT_P4, FSM_VARIANT_P8, FSM_VARIANT_B, FSM_VARIANT_G = -1, 0, 1, 2, 3
 FSM_VARIANT_HS, FSM_VARIANT_CL, FSM_VARIANT_N8, FSM_VARIANT_R16 = 5, 6, 7, 8
-VARIANT_NAMES = {0: "P4", 1: "P8", 2: "B", 3: "G", 4: "H8", 5: "HS", 6: "CL", 7: "N8", 8: "R16"}
+VARIANT_NAMES = {0: "P4", 1: "P8", 2: "B", 3: "G", 5: "HS", 6: "CL", 7: "N8", 8: "R16"}
 FSM_MERGE_PARALLEL, FSM_MERGE_SEQUENTIAL = 0, 1
 FSM_EAGER_OFF = 1
+FSM_PRERESOLVE_NONE = 0x80000000
 
 # every symbol declared in include/fsmspec.h
 EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_set_stream",
            "fsm_run_spec_k", "fsm_run_spec_k_async", "fsm_run_spec_k_host", "fsm_set_options",
            "fsm_get_options", "fsm_get_stats", "fsm_run_shard", "fsm_shard_fixup", "fsm_shard_free",
-           "fsm_map_compose", "fsm_lookback_table", "fsm_version", "fsm_autotune", "fsm_run_multi")
+           "fsm_map_compose", "fsm_compose_from", "fsm_lookback_table", "fsm_version", "fsm_autotune",
+           "fsm_run_multi", "fsm_debug_set_spec", "fsm_debug_get_merge")
 
 
 class fsm_options(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
                 ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32),
-                ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32)]
+                ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32), ("preresolve", ctypes.c_uint32),
+                ("grid_sms", ctypes.c_uint32)]
 
 
 class fsm_tuning(ctypes.Structure):
@@ -45,8 +48,12 @@ class fsm_tuning(ctypes.Structure):
 class fsm_stats(ctypes.Structure):
     _fields_ = [("chunks", ctypes.c_uint64), ("tiles", ctypes.c_uint64), ("reexec_chunks", ctypes.c_uint64),
                 ("reexec_symbols", ctypes.c_uint64), ("boundary_misses", ctypes.c_uint64),
+                ("reexec_true", ctypes.c_uint64), ("reexec_true_symbols", ctypes.c_uint64),
+                ("reexec_candidate", ctypes.c_uint64), ("reexec_candidate_symbols", ctypes.c_uint64),
+                ("eager_resolved", ctypes.c_uint64), ("max_miss_chain", ctypes.c_uint64),
                 ("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
-                ("variant", ctypes.c_uint32), ("k_slots", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32)]
+                ("variant", ctypes.c_uint32), ("k_slots", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32),
+                ("preresolve", ctypes.c_uint32)]
 
 
 class fsm_shard_map(ctypes.Structure):
@@ -57,6 +64,25 @@ class fsm_shard_map(ctypes.Structure):
     def slots(self):
         return [(int(self.start[s]), int(self.end[s]), int(self.count[s]))
                 for s in range(FSM_KMAX) if (self.valid_mask >> s) & 1]
+
+
+_L6 = ctypes.c_uint32 * FSM_KMAX * 32 * 6
+
+
+class fsm_debug_merge(ctypes.Structure):
+    _fields_ = [("k", ctypes.c_uint32), ("start", _L6), ("end", _L6), ("count", _L6), ("brk", _L6),
+                ("identity", ctypes.c_uint32 * 32 * 6)]
+
+    def mapping(self, level: int, lane: int) -> dict:
+        """Slot s -> (start, end, count) for valid slots, (start, None, brk) for invalid ones."""
+        out = {}
+        for s in range(self.k):
+            st = int(self.start[level][lane][s])
+            if st == 0xFFFFFFFF:
+                continue
+            b = int(self.brk[level][lane][s])
+            out[st] = (int(self.end[level][lane][s]), int(self.count[level][lane][s])) if b == 0xFFFFFFFF else None
+        return out
 
 
 class FsmError(RuntimeError):
@@ -101,6 +127,10 @@ def lib() -> ctypes.CDLL:
                                        ctypes.POINTER(fsm_shard_map)]),
             "fsm_lookback_table": (_I32, [_P, _U32, _U32, _U32, _P, _P]),
             "fsm_version": (ctypes.c_char_p, []),
+            "fsm_compose_from": (_I32, [ctypes.POINTER(fsm_shard_map), _U32, _U32, _U64, ctypes.POINTER(_U32),
+                                        ctypes.POINTER(_U64), ctypes.POINTER(_U32)]),
+            "fsm_debug_set_spec": (_I32, [_P, _P, _U32, _U32, _U32]),
+            "fsm_debug_get_merge": (_I32, [_P, ctypes.POINTER(fsm_debug_merge)]),
             "fsm_run_multi": (_I32, [ctypes.POINTER(_P), _U32, _P, _U64, ctypes.POINTER(_U32), ctypes.POINTER(_U32),
                                      ctypes.POINTER(_U64)]),
             "fsm_autotune": (_I32, [_P, _P, _U64, _U32, _U32, _U64, ctypes.POINTER(fsm_tuning)]),
@@ -148,6 +178,17 @@ def map_compose(a: fsm_shard_map, b: fsm_shard_map) -> fsm_shard_map:
     return out
 
 
+def compose_from(maps, start_state: int, start_count: int = 0) -> tuple[int, int, int]:
+    """fsm_compose_from (host only): follow start_state through the shard maps in order ->
+    (state, count, first_miss) with first_miss == len(maps) when every map matched."""
+    n = len(maps)
+    arr = (fsm_shard_map * max(n, 1))(*maps)
+    q, c, g = _U32(), _U64(), _U32()
+    _check(lib().fsm_compose_from(arr, n, start_state, start_count, ctypes.byref(q), ctypes.byref(c), ctypes.byref(g)),
+           "fsm_compose_from")
+    return int(q.value), int(c.value), int(g.value)
+
+
 class FSM:
     """One handle = one DFA on the current CUDA device (fsm_create_ex)."""
 
@@ -187,8 +228,9 @@ class FSM:
 
     def set_options(self, chunk_bytes: int = 0, threads_per_tile: int = 0, variant: int = FSM_VARIANT_AUTO,
                     merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0, lookback_len: int = 0,
-                    eager_window: int = 0) -> None:
-        o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm, lookback_len, eager_window)
+                    eager_window: int = 0, preresolve: int = 0, grid_sms: int = 0) -> None:
+        o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm, lookback_len, eager_window,
+                        preresolve, grid_sms)
         _check(lib().fsm_set_options(self._h, ctypes.byref(o)), "fsm_set_options")
 
     def options(self) -> dict:
@@ -237,6 +279,26 @@ class FSM:
                                    halo_len, k, ctypes.byref(m), ctypes.byref(st) if keep else None),
                "fsm_run_shard")
         return m, (Shard(st) if keep else None)
+
+    # ------------------------------------------------------------------------- test-only hooks
+    def debug_set_spec(self, sets, chunk_bytes: int, k: int = 0) -> None:
+        """fsm_debug_set_spec: fixed chunk_bytes geometry; ``sets`` = per-chunk speculated state lists
+        (None = look-back as usual; an entry None / missing = no state in that slot)."""
+        if sets is None:
+            _check(lib().fsm_debug_set_spec(self._h, None, 0, 0, chunk_bytes), "fsm_debug_set_spec")
+            return
+        k = k or max(len(x) for x in sets)
+        a = np.full((len(sets), k), 0xFFFFFFFF, np.uint32)
+        for j, x in enumerate(sets):
+            for s, v in enumerate(x):
+                if v is not None:
+                    a[j, s] = v
+        _check(lib().fsm_debug_set_spec(self._h, a.ctypes.data, len(sets), k, chunk_bytes), "fsm_debug_set_spec")
+
+    def debug_get_merge(self) -> fsm_debug_merge:
+        m = fsm_debug_merge()
+        _check(lib().fsm_debug_get_merge(self._h, ctypes.byref(m)), "fsm_debug_get_merge")
+        return m
 
     def shard_fixup(self, shard: "Shard", true_start: int) -> tuple[int, int]:
         q, n = _U32(), _U64()

@@ -1,0 +1,202 @@
+"""The paper's worked examples replayed on the CUDA merge, through the
+test-only hook fsm_debug_set_spec (fixed tiny chunks, injected speculated sets) and the merge-tree
+readback fsm_debug_get_merge, plus the per-run re-execution counters.
+
+* Fig. 2: chunks `/*xx` | `x**/`, spec-1; look-back on `x` guesses a, chunk 1 ends in b,
+  the check fails, chunk 1 is re-executed from c; final a; 1 re-execution.
+* Fig. 4: four chunks of two bytes, spec-2 with the figure's sets injected;
+  merged chunks 0+1 = {a->c, c->c}; merged 2+3 = {c->a, a invalid}; root = {a->a, c->a}; the
+  delayed strategy re-executes nothing, nor does the sequential merge (Fig. 4a).
+Expected values come from tests/golden/c_comment_fig2_fig4.json (the paper's narrative)."""
+import numpy as np
+import pytest
+
+from fsmgen import dfas, streams
+from oracle import seq, speck
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from paper_conf_ppopp_xiaja20_b200 import fsmspec  # noqa: E402
+from paper_conf_ppopp_xiaja20_b200.fsmspec import FSM  # noqa: E402
+
+ST = {"a": 0, "b": 1, "c": 2, "d": 3}
+NAME = {v: k for k, v in ST.items()}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8}
+
+
+def dev(data: np.ndarray):
+    buf = torch.zeros(data.size + 64, dtype=torch.uint8, device="cuda")
+    buf[:data.size] = torch.from_numpy(np.ascontiguousarray(data))
+    return buf, buf.data_ptr()
+
+
+def named(m, level, lane):
+    """Level/lane mapping of the readback in the golden file's notation."""
+    return {NAME[s]: (None if v is None else [NAME[v[0]], v[1]]) for s, v in m.mapping(level, lane).items()}
+
+
+@pytest.mark.parametrize("var", list(VARIANTS))
+def test_fig2_speculation_and_reexecution(golden, var):
+    g = golden["c_comment_fig2_fig4"]["P2"]
+    d = dfas.c_comment(True)
+    data = np.frombuffer("".join(g["chunks"]).encode(), np.uint8)
+    with FSM.from_dfa(d) as f:
+        f.set_options(variant=VARIANTS[var], eager_window=fsmspec.FSM_EAGER_OFF)
+        f.debug_set_spec(None, chunk_bytes=len(g["chunks"][0]))
+        buf, ptr = dev(data)
+        got = f.run_spec_k(ptr, data.size, 1)
+        st = f.stats()
+        m = f.debug_get_merge()
+    assert got == (ST[g["final"]], 1) == seq.run(d, data)
+    assert named(m, 0, 0) == {"a": ["c", 0]}                     # chunk 0 from the known start a
+    assert named(m, 0, 1) == {g["guess_chunk1"]: ["b", 3]}       # look-back on x guesses a; ends in b
+    assert named(m, 1, 0) == {"a": None}                         # c is not a speculated start: invalid
+    assert m.brk[1][0][0] == 1 and m.end[1][0][0] == ST["c"]     # ... when entering chunk 1 in state c
+    assert st["reexec_true"] == g["reexec"] and st["reexec_candidate"] == 0
+    assert st["reexec_true_symbols"] == 4 and st["max_miss_chain"] == 1
+
+
+@pytest.mark.parametrize("var", list(VARIANTS))
+def test_fig4_merge_tree(golden, var):
+    g = golden["c_comment_fig2_fig4"]["P3"]
+    d = dfas.c_comment(True)
+    data = np.frombuffer("".join(g["chunks"]).encode(), np.uint8)
+    sets = [[ST[s] for s in ss] for ss in g["injected_sets"]]
+    with FSM.from_dfa(d) as f:
+        f.set_options(variant=VARIANTS[var])
+        f.debug_set_spec(sets, chunk_bytes=2)
+        buf, ptr = dev(data)
+        got = f.run_spec_k(ptr, data.size, 2)
+        st = f.stats()
+        m = f.debug_get_merge()
+    assert got == (ST["a"], 1) == seq.run(d, data)
+    # level 0: the chunk mappings of Fig. 4, counts with F = {a}
+    assert named(m, 0, 0) == {"a": ["c", 0], "c": ["d", 0]}
+    assert named(m, 0, 1) == {"c": ["c", 0], "d": ["c", 0]}
+    assert named(m, 0, 2) == {"a": ["a", 2], "c": ["d", 0]}
+    assert named(m, 0, 3) == {"c": ["a", 1], "d": ["a", 1]}
+    # level 1 = the pairwise merges, level 2 = the root (Fig. 4b)
+    assert named(m, 1, 0) == g["merged_01"]
+    assert named(m, 1, 2) == g["merged_23"]
+    a_slot = sets[2].index(ST["a"])
+    assert m.brk[1][2][a_slot] == 3 and m.end[1][2][a_slot] == ST["a"]  # invalid entering chunk 3 in a
+    assert named(m, 2, 0) == g["root"]
+    assert all(m.identity[0][lane] for lane in range(4, 32)) and not any(m.identity[0][:4])
+    # P4: the delayed strategy re-executes nothing
+    assert st["reexec_chunks"] == golden["c_comment_fig2_fig4"]["P4"]["reexec_delayed"] == 0
+    assert st["boundary_misses"] == 0
+
+
+def test_fig4_sequential_merge_reexecutes_nothing(golden):
+    g = golden["c_comment_fig2_fig4"]
+    d = dfas.c_comment(True)
+    data = np.frombuffer("".join(g["P3"]["chunks"]).encode(), np.uint8)
+    sets = [[ST[s] for s in ss] for ss in g["P3"]["injected_sets"]]
+    with FSM.from_dfa(d) as f:
+        f.set_options(merge=fsmspec.FSM_MERGE_SEQUENTIAL)
+        f.debug_set_spec(sets, chunk_bytes=2)
+        buf, ptr = dev(data)
+        assert f.run_spec_k(ptr, data.size, 2) == (ST["a"], 1)
+        assert f.stats()["reexec_chunks"] == g["P4"]["reexec_sequential"]
+
+
+def test_injected_chunk0_without_true_start_is_resolved():
+    """Chunk 0's injected set does not contain q0 = a: the true path misses at chunk 0 and is
+    re-executed (a tile-boundary miss of tile 0), the result is still exact."""
+    d = dfas.c_comment(True)
+    data = np.frombuffer(b"/*xxx**/", np.uint8)
+    with FSM.from_dfa(d) as f:
+        f.debug_set_spec([[ST["c"], ST["d"]], [ST["c"], ST["d"]], [ST["a"], ST["c"]], [ST["c"], ST["d"]]], chunk_bytes=2)
+        buf, ptr = dev(data)
+        assert f.run_spec_k(ptr, data.size, 2) == (ST["a"], 1)
+        st = f.stats()
+    assert st["boundary_misses"] == 1 and st["reexec_true"] >= 1
+
+
+def test_debug_hook_validates():
+    d = dfas.c_comment(True)
+    with FSM.from_dfa(d) as f:
+        with pytest.raises(fsmspec.FsmError):
+            f.debug_set_spec([[0, 0]], chunk_bytes=2)        # duplicated slot (reading A6)
+        with pytest.raises(fsmspec.FsmError):
+            f.debug_set_spec([[7]], chunk_bytes=2)           # not a state
+        f.debug_set_spec([[0], [0]], chunk_bytes=4)
+        buf, ptr = dev(np.frombuffer(b"/*xxx**/x", np.uint8))
+        with pytest.raises(fsmspec.FsmError):
+            f.run_spec_k(ptr, 9, 1)                         # 3 chunks, 2 injected
+        f.debug_set_spec(None, 0)                           # cleared: normal geometry again
+        assert f.run_spec_k(ptr, 9, 1) == seq.run(d, np.frombuffer(b"/*xxx**/x", np.uint8))
+
+
+# --------------------------------------------------------------------- per-run counters (a8)
+def _true_path_misses(d, data, chunk, k):
+    """#chunks whose true start is not in their depth-1 look-back set (A5), chunk 0 = {q0}: what
+    the delayed strategy must re-execute, from the oracle loop per chunk."""
+    x, miss = d.start, 0
+    for j, b in enumerate(range(0, data.size, chunk)):
+        if j and x not in speck.lookback(d.table, int(data[b - 1]), k):
+            miss += 1
+        x = seq.run_from(d, x, data[b:b + chunk])[0]
+    return miss
+
+
+@pytest.mark.parametrize("n,m,k,pre", [(8, 3, 1, 0), (8, 4, 2, 0), (8, 4, 2, fsmspec.FSM_PRERESOLVE_NONE),
+                                       (16, 5, 3, 1), (16, 5, 3, 0), (64, 6, 4, 2)])
+def test_reexec_true_equals_model_miss_count(n, m, k, pre):
+    d = dfas.random_dfa(n, m, seed=300 + n + m)
+    data = streams.splitmix_bytes(41 + n, 0, 1 << 20)
+    chunk = 256
+    with FSM.from_dfa(d) as f:
+        f.set_options(chunk_bytes=chunk, eager_window=fsmspec.FSM_EAGER_OFF, preresolve=pre)
+        buf, ptr = dev(data)
+        assert f.run_spec_k(ptr, data.size, k) == seq.run(d, data)
+        st = f.stats()
+    assert st["reexec_true"] == _true_path_misses(d, data, chunk, k), st
+    assert st["reexec_chunks"] == st["reexec_true"] + st["reexec_candidate"]
+    if pre == fsmspec.FSM_PRERESOLVE_NONE:
+        assert st["reexec_candidate"] == 0      # only the true path is ever re-executed
+
+
+def test_stats_are_per_run():
+    """Counters describe the most recent call: three async runs on other inputs, then a sync run,
+    give the same counters as a fresh handle's single sync run (no leak across runs)."""
+    d = dfas.random_dfa(8, 4, seed=77)
+    data = streams.splitmix_bytes(77, 0, 3 << 20)
+    other = streams.splitmix_bytes(78, 0, 5 << 20)
+    with FSM.from_dfa(d) as f:
+        f.set_options(eager_window=fsmspec.FSM_EAGER_OFF)
+        buf, ptr = dev(data)
+        f.run_spec_k(ptr, data.size, 2)
+        fresh = f.stats()
+    assert fresh["reexec_chunks"] > 0
+    with FSM.from_dfa(d) as f:
+        f.set_options(eager_window=fsmspec.FSM_EAGER_OFF)
+        buf, ptr = dev(data)
+        obuf, optr = dev(other)
+        res = torch.zeros(4, dtype=torch.int32, device="cuda")
+        for _ in range(3):
+            f.run_spec_k_async(optr, other.size, 2, res.data_ptr())
+        f.run_spec_k(ptr, data.size, 2)
+        assert f.stats() == fresh
+        # an async run's own counters are readable too
+        f.run_spec_k_async(optr, other.size, 2, res.data_ptr())
+        a1 = f.stats()
+        f.run_spec_k_async(optr, other.size, 2, res.data_ptr())
+        assert f.stats() == a1
+
+
+def test_unaligned_input_peels_one_sector():
+    """An unaligned pointer runs from the aligned address below it (chunk 0 = [head, chunk)); the
+    result and the re-execution counters do not depend on the offset beyond chunk 0."""
+    d = dfas.random_dfa(8, 2, seed=5)
+    data = streams.splitmix_bytes(5, 0, (8 << 20) + 77)
+    exp = seq.run(d, data)
+    for off in (0, 1, 7, 31):
+        buf = torch.zeros(data.size + 128, dtype=torch.uint8, device="cuda")
+        buf[off:off + data.size] = torch.from_numpy(data)
+        with FSM.from_dfa(d) as f:
+            for lb in (0, 64):
+                f.set_options(lookback_len=lb)
+                for k in (1, 2):
+                    assert f.run_spec_k(buf.data_ptr() + off, data.size, k) == exp, (off, lb, k)

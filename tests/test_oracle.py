@@ -206,6 +206,44 @@ def test_random_dfa_image_size(n, m):
         assert len(set(d.table[:, c].tolist())) == m
 
 
+def _mod7_bytes_dfa():
+    """Byte-mode Div7: state = value of the big-endian byte string so far mod 7, F = {0}."""
+    t = np.array([[(256 * s + c) % 7 for c in range(256)] for s in range(7)], np.uint32)
+    acc = np.zeros(7, np.uint8)
+    acc[0] = 1
+    return dfas.DFA(t, 0, acc, False, "mod7_bytes")
+
+
+@pytest.mark.parametrize("G,piece", [(1, 1 << 28), (5, 64), (9, 1000)])
+def test_certify_closed_form(G, piece):
+    """seq.certify against the closed form of byte-mode Div7: claims computed with
+    Python big ints (int.from_bytes(prefix) % 7) pass and return (value mod 7, #prefixes = 0 mod
+    7); a corrupted claim, a wrong segment-0 start, or a claim off by one segment all fail."""
+    d = _mod7_bytes_dfa()
+    data = np.random.default_rng(G).integers(0, 256, 3001).astype(np.uint8)
+    L = data.size
+    bounds = [L * g // G for g in range(G)] + [L]
+    val = [int.from_bytes(data[:b].tobytes(), "big") % 7 for b in range(L + 1)]
+    claims = [val[b] for b in bounds[:-1]]
+    exp = (val[L], sum(1 for i in range(1, L + 1) if val[i] == 0))
+
+    def fetch(lo, hi):
+        return data[lo:hi]
+
+    assert seq.certify(d, bounds, claims, fetch, piece=piece) == exp
+    if G > 1:
+        bad = list(claims)
+        bad[G // 2] = (bad[G // 2] + 1) % 7
+        with pytest.raises(seq.CertificateError):
+            seq.certify(d, bounds, bad, fetch, piece=piece)
+        shifted = [claims[0]] + [val[b + 1] for b in bounds[1:-1]]
+        if shifted != claims:
+            with pytest.raises(seq.CertificateError):
+                seq.certify(d, bounds, shifted, fetch, piece=piece)
+    with pytest.raises(seq.CertificateError):
+        seq.certify(d, bounds, [(claims[0] + 3) % 7] + claims[1:], fetch, piece=piece)
+
+
 def test_splitmix_c_matches_numpy():
     w = streams.splitmix_words(123, 5, 100)
     b = streams.splitmix_bytes(123, 40, 800)

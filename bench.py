@@ -205,6 +205,23 @@ def run_reference(args, w):
     print(json.dumps(line), flush=True)
 
 
+def config_key(args, w):
+    """Key of this workload in profiles/ncu_metrics.json (the ncu capture of the same config)."""
+    if args.config == "c5":
+        return f"c5_n{args.n_states}_m{args.m}_k{w['k']}"
+    return f"{args.config}_k{w['k']}" + (f"_ac{args.ac_states}" if args.config == "c3" else "")
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def config_json(args, w):
     return {"workload": w["name"], "input_bytes": w["total"], "k": w["k"], "lookback_len": w.get("lookback"),
             "eager_window": w.get("eager", 0),
@@ -449,9 +466,14 @@ def main():
     except OSError:
         pass
     peak = float(peaks.get("hbm_gbs", 6650.0))
-    traffic = None
-    if args.config == "c5" and args.n_states == 8 and args.m == 2 and args.k == 2:
-        traffic = round(1.037 * n)   # per launch: dram read+write / input bytes of the committed ncu capture
+    # per-launch DRAM traffic, LDS utilisation and bank conflicts from the committed ncu capture of
+    # the same config (profiles/ncu_metrics.json, written by tools/ncu_metrics.py), scaled per byte
+    nm = {}
+    try:
+        nm = json.load(open(os.path.join(ROOT, "profiles", "ncu_metrics.json"))).get(config_key(args, w), {})
+    except (OSError, ValueError):
+        pass
+    traffic = round(nm["dram_bytes_per_input_byte"] * n) if nm.get("dram_bytes_per_input_byte") else None
     line = {
         "metric": METRIC, "value": round(gbs, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(step_s * 1e3, 4), "higher_is_better": True,
@@ -460,13 +482,17 @@ def main():
         "roofline": {"bound": "hbm", "achieved": round(n / step_s / 1e9, 3) if world == 1 else round(gbs / world, 3),
                      "peak": peak, "unit": "GB/s", "frac": round((n / step_s / 1e9) / peak, 4),
                      "traffic": traffic, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if peaks else "fallback"},
-        "traffic_note": "ncu --set full (profiles/r01_ncu_c5_n8m2k2_8GiB.txt): dram read+write = 1.037 x input bytes (8.881 GB read + 0.030 GB written for 8 GiB)",
+        "ncu": ({"source": nm.get("source"), "capture_input_bytes": nm.get("input_bytes"),
+                 "dram_bytes_per_input_byte": nm.get("dram_bytes_per_input_byte"), "lds_util": nm.get("lds_util"),
+                 "bank_conflicts_per_kib": nm.get("bank_conflicts_per_kib"), "alu_pipe_pct": nm.get("alu_pipe_pct"),
+                 "issue_pct": nm.get("issue_pct")} if nm else None),
         "clocks": clk.summary(),
         # one fused kernel per step, plus the look-back window pre-pass when the window is >= 32 bytes
         # (and, for N > 1, a fix-up kernel per shard-boundary miss round)
         "gpu_launches": args.steps * (2 if (lookback or 0) >= 32 else 1),
         "result": {"final_state": final[0], "accept_count": final[1]},
         "stats": {kk: v for kk, v in st.items()},
+        "reexec_rate": round(st["reexec_true"] / st["chunks"], 6) if st.get("chunks") else None,
         "e2e": e2e,
     }
     if tuning is not None:
@@ -527,6 +553,7 @@ def main():
                                 "sample": f"first {cb['bytes']} bytes of the workload ({cb['seconds']:.1f} s)"}
         line["parity_sample"] = {"bytes": cb["bytes"], "ok": gp == cb["result"]}
         line["host_cores"] = os.cpu_count()
+        line["cpu_model"] = cpu_model()
         if "host" in w and not args.no_certify:
             line["parity_full"] = certify_full(args, w, f, buf, n, k, final)
     print(json.dumps(line), flush=True)

@@ -155,10 +155,16 @@ typedef struct {
     uint32_t grid_sms;          /* SMs the persistent grids use (0 = all): the grid-size sweep of the
                                    sequential- vs parallel-merge ablation (Figs. 7-11 vary the number of
                                    thread blocks) */
+    uint32_t check;             /* runtime membership check of the merge: FSM_CHECK_AUTO (default),
+                                   FSM_CHECK_NESTED = Alg. 1 (O(k^2)), FSM_CHECK_HASH = Alg. 2
+                                   (O(k), per-thread shared-memory buckets); the hash form is
+                                   built for k > 8 (instantiated K = 12, 16) and falls back to Alg. 1
+                                   where its scratch does not fit next to the table.  Identical results. */
 } fsm_options;
 
 #define FSM_EAGER_OFF 1u
 #define FSM_PRERESOLVE_NONE 0x80000000u
+enum { FSM_CHECK_AUTO = 0, FSM_CHECK_NESTED = 1, FSM_CHECK_HASH = 2 };
 
 int fsm_set_options(fsm_t *f, const fsm_options *opt);
 int fsm_get_options(const fsm_t *f, fsm_options *opt);
@@ -182,6 +188,7 @@ typedef struct {
     uint64_t eager_resolved;    /* true-path misses completed from an eager-completion entry (NEXT-3) */
     uint64_t max_miss_chain;    /* longest run of consecutive re-executed chunks on the true path */
     uint32_t chunk_bytes, threads_per_tile, variant, k_slots, lookback_len, preresolve;
+    uint32_t check;             /* FSM_CHECK_NESTED or FSM_CHECK_HASH: the check the run used */
 } fsm_stats;
 
 /* Synchronises the handle's stream (the counters live on the device). */
@@ -279,7 +286,8 @@ int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k_min, u
  * variant and instantiated K share one persistent grid, whose CTAs take (tile, DFA) pairs in
  * tile-major order so that the input is read from HBM about once per group (the other DFAs hit
  * the tile in L2).  Each handle's own options (look-back, eager window) apply; the chunk and tile
- * geometry are the first handle of each group's.
+ * geometry are the first handle of each group's.  DFAs run with k > 8 are not fused (one launch
+ * each, same results).
  *   fsms, m        1 <= m <= FSM_MULTI_MAX distinct handles, same input mode and device; the work is
  *                  enqueued on fsms[0]'s stream
  *   input, len     as fsm_run_spec_k (one input for all)

@@ -39,7 +39,7 @@ typedef void (*MultiFn)(Params, const Params *, uint32_t);
 // Kernel instantiations live in one translation unit per table variant (kernels_*.cu, compiled in
 // parallel); each exports these accessors.
 #define FSM_DECLARE_VARIANT(NAME)                                   \
-    KernelFn get_kernel_##NAME(int K, bool split);                  \
+    KernelFn get_kernel_##NAME(int K, bool split, bool hash);       \
     MultiFn get_multi_##NAME(int K);                                \
     FixFn get_fix_##NAME();                                         \
     void get_seq_##NAME(int K, SeqLocalFn &l, SeqWalkFn &w);       \
@@ -53,17 +53,17 @@ FSM_DECLARE_VARIANT(cl)
 FSM_DECLARE_VARIANT(n8)
 FSM_DECLARE_VARIANT(r16)
 
-static KernelFn get_kernel(int var, int K, bool split)
+static KernelFn get_kernel(int var, int K, bool split, bool hash)
 {
     switch (var) {
-    case VAR_P4: return get_kernel_p4(K, split);
-    case VAR_P8: return get_kernel_p8(K, split);
-    case VAR_HS: return get_kernel_hs(K, split);
-    case VAR_CL: return get_kernel_cl(K, split);
-    case VAR_N8: return get_kernel_n8(K, split);
-    case VAR_R16: return get_kernel_r16(K, split);
-    case VAR_B: return get_kernel_b(K, split);
-    default: return get_kernel_g(K, split);
+    case VAR_P4: return get_kernel_p4(K, split, hash);
+    case VAR_P8: return get_kernel_p8(K, split, hash);
+    case VAR_HS: return get_kernel_hs(K, split, hash);
+    case VAR_CL: return get_kernel_cl(K, split, hash);
+    case VAR_N8: return get_kernel_n8(K, split, hash);
+    case VAR_R16: return get_kernel_r16(K, split, hash);
+    case VAR_B: return get_kernel_b(K, split, hash);
+    default: return get_kernel_g(K, split, hash);
     }
 }
 static MultiFn get_multi(int var, int K)
@@ -175,6 +175,7 @@ struct fsm {
     size_t seq_cap = 0;
     // geometry / configuration of the most recent run (the counters are read from d_stats)
     fsm_stats last{};
+    uint32_t last_head = 0;  // peeled head of the most recent run (kernel coordinates)
     // test hook (fsm_debug_set_spec): fixed chunk bytes, injected sets, merge-tree readback
     uint32_t dbg_chunk = 0, dbg_n = 0, dbg_k = 0;
     uint16_t *d_dbg_spec = nullptr;
@@ -190,6 +191,10 @@ struct fsm_shard {
     uint32_t k = 0;
     int variant = 0;           // the table variant the shard ran with (the fix-up uses the same)
     fsm_shard_map map{};
+    // keyed runs: the tile descriptors (aggregates A_t, prefixes P_t) the fix-up walks
+    TileDesc *d_desc = nullptr;
+    uint32_t ntiles = 0, head = 0;
+    uint64_t tile_bytes = 0;
 };
 
 #define CK(x)                                                  \
@@ -439,12 +444,14 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
     if (o->eager_window > FSM_EAGER_OFF && (o->eager_window % 32 || o->eager_window > kExtWindow)) return FSM_EINVAL;
     if (o->preresolve > FSM_KMAX && o->preresolve != FSM_PRERESOLVE_NONE) return FSM_EINVAL;
+    if (o->check > FSM_CHECK_HASH) return FSM_EINVAL;
     f->opt.chunk_bytes = o->chunk_bytes;            // 0 = adaptive
     f->opt.threads_per_tile = o->threads_per_tile;  // 0 = auto
     f->opt.variant = o->variant;
     f->opt.merge = o->merge;
     f->opt.ctas_per_sm = o->ctas_per_sm;
     f->opt.grid_sms = o->grid_sms;
+    f->opt.check = o->check;
     f->opt.lookback_len = o->lookback_len;
     f->opt.eager_window = o->eager_window;
     f->opt.preresolve = o->preresolve;
@@ -497,8 +504,13 @@ struct RunSpec {
     bool accumulate = false;                // keep the counters of the call's earlier launches
 };
 
+constexpr int kMultiMaxK = 8;  // fused multi-FSM kernels are instantiated for K <= 8
+// FSM_CHECK_AUTO: Alg. 2 for K >= 12 when its per-thread columns fit next to the table at the full
+// tile size, else Alg. 1 (measured on B200: the hash form wins where the tile keeps
+// its size, e.g. 64-state B k = 16 +12 %, and loses where the tile must halve, e.g. HTML CL -26 %)
+constexpr bool kHashAuto = true;
 // R5 default (fsm_options.preresolve = 0): see DESIGN.md "R5".
-constexpr uint32_t kPreresolveDefault = FSM_KMAX;
+constexpr uint32_t kPreresolveDefault = 1;
 static uint32_t preresolve_of(const fsm *f)
 {
     const uint32_t v = f->opt.preresolve;
@@ -566,7 +578,17 @@ struct Prepared {
     uint32_t T;
     size_t smem;
     bool split;
+    bool hash;  // Alg. 2 runtime check (K >= 12)
 };
+
+// Alg. 1 vs Alg. 2 (fsm_options.check = FSM_CHECK_AUTO): see DESIGN.md "a5"
+static bool hash_wanted(const fsm *f, int K)
+{
+    if (K < 12) return false;
+    if (f->opt.check == FSM_CHECK_HASH) return true;
+    if (f->opt.check == FSM_CHECK_NESTED) return false;
+    return kHashAuto;
+}
 
 static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
 {
@@ -601,9 +623,17 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     if (r.merge == FSM_MERGE_SEQUENTIAL) T = std::min<uint32_t>(T, kThreads);
     if (split_kernel(var, K) && T < 64) T = 64;  // at least one worker warp besides the epilogue warp
     bool split = split_kernel(var, K) && !r.multi && r.merge == FSM_MERGE_PARALLEL;
-    if (split) {  // the double-buffered layout must fit next to the table (HS sizes its hot rows after)
+    bool hash = hash_wanted(f, K) && !r.multi && r.merge == FSM_MERGE_PARALLEL;
+    if (hash) split = false;  // Alg. 2 kernels are instantiated unsplit
+    {
         const uint32_t tb = var == VAR_HS ? 0u : f->img_bytes[var];
-        split = Layout(T, K, scratch_offset(var, tb), true).total <= kMaxSmem;
+        if (hash && !f->opt.threads_per_tile && f->opt.check == FSM_CHECK_HASH) {
+            // Alg. 2 requested: halve the tile until its per-thread columns fit next to the table
+            while (T > 64 && Layout(T, K, scratch_offset(var, tb), false, true).total > kMaxSmem) T >>= 1;
+        }
+        if (hash && Layout(T, K, scratch_offset(var, tb), false, true).total > kMaxSmem) hash = false;  // Alg. 1
+        if (split)  // the double-buffered layout must fit next to the table (HS sizes its hot rows after)
+            split = Layout(T, K, scratch_offset(var, tb), true, hash).total <= kMaxSmem;
     }
     const uint64_t tile_bytes = (uint64_t)tile_chunks(T, split) * chunk;
     uint64_t ntiles64 = (len_bytes + tile_bytes - 1) / tile_bytes;
@@ -664,13 +694,13 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
 
     if (var == VAR_HS) {
         // as many hot rows as fit next to this launch's scratch (227 KB per CTA)
-        const uint32_t scratch = Layout(T, K, 0, split).total;
+        const uint32_t scratch = Layout(T, K, 0, split, hash).total;
         const uint32_t avail = scratch < kMaxSmem ? kMaxSmem - scratch : 0u;
         const uint32_t hot = std::min<uint32_t>(f->hot_rows, avail / 512);
         p.hot_rows = hot;
         p.table_bytes = hot * 512;
     }
-    const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes), split).total;
+    const size_t smem = Layout(T, K, scratch_offset(var, p.table_bytes), split, hash).total;
 
     if (p.lookback >= 32) {
         // a3 pre-pass: ranked look-back candidates per chunk (spec_kernel.cuh)
@@ -703,6 +733,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     out.T = T;
     out.smem = smem;
     out.split = split;
+    out.hash = hash;
     if (r.merge == FSM_MERGE_SEQUENTIAL) return FSM_OK;
     if ((rc = ensure_desc(f, ntiles))) return rc;
     out.p.desc = f->d_desc;
@@ -717,6 +748,8 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     f->last.k_slots = K;
     f->last.lookback_len = p.lookback;
     f->last.preresolve = p.preresolve;
+    f->last_head = head;
+    f->last.check = hash ? FSM_CHECK_HASH : FSM_CHECK_NESTED;
     return FSM_OK;
 }
 
@@ -735,7 +768,7 @@ static int launch_run(fsm *f, const RunSpec &r)
         return launch_seq(f, p, var, K, T);
     }
 
-    KernelFn fn = get_kernel(var, K, pr.split);
+    KernelFn fn = get_kernel(var, K, pr.split, pr.hash);
     CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)T, smem));
@@ -938,6 +971,18 @@ extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const
         st->k = k;
         st->variant = (int)f->last.variant;
         st->map = m;
+        if (keyed && f->last.tiles) {
+            st->ntiles = (uint32_t)f->last.tiles;
+            st->tile_bytes = (uint64_t)f->last.threads_per_tile * f->last.chunk_bytes;
+            st->head = f->last_head;
+            if (cudaMalloc(&st->d_desc, st->ntiles * sizeof(TileDesc)) != cudaSuccess ||
+                cudaMemcpyAsync(st->d_desc, f->d_desc, st->ntiles * sizeof(TileDesc), cudaMemcpyDeviceToDevice,
+                                f->stream) != cudaSuccess ||
+                cudaStreamSynchronize(f->stream) != cudaSuccess) {
+                fsm_shard_free(st);
+                return FSM_ECUDA;
+            }
+        }
         *state = st;
     }
     return FSM_OK;
@@ -952,52 +997,75 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
             *count = st->map.count[s];
             return FSM_OK;
         }
+    CK(cudaMemsetAsync(f->d_stats, 0, sizeof(DevStats), f->stream));  // the fix-up's own counters
     const bool bits = f->mode == FSM_INPUT_BITS_MSB;
     const uint64_t whole = bits ? st->len / 8 : st->len;
     const int var = st->variant;
-    FixParams fp{};
-    fp.in = st->input;
-    fp.len = whole;
-    fp.limit = (uint64_t)1 << 20;
-    fp.table = f->d_img[var];
-    fp.n_states = f->dfa.n;
-    fp.x = to_int(f, true_start);
-    fp.k = st->map.k;
-    fp.valid_mask = st->map.valid_mask;
-    for (int s = 0; s < KMAX; s++) {
-        const bool v = (st->map.valid_mask >> s) & 1u;
-        fp.start[s] = v ? to_int(f, st->map.start[s]) : st->map.start[s];
-        fp.end[s] = v ? to_int(f, st->map.end[s]) : st->map.end[s];
-        fp.count[s] = st->map.count[s];
+    uint32_t y = to_int(f, true_start);
+    uint64_t cy = 0, resume_byte = 0;
+    if (st->d_desc && st->ntiles) {
+        // walk x's path over the keyed run's tile descriptors (fixup_kernel.cuh)
+        FixParams fp{};
+        fp.in = st->input;
+        fp.len = whole;
+        fp.head = st->head;
+        fp.tile_bytes = st->tile_bytes;
+        fp.ntiles = st->ntiles;
+        fp.limit = (uint64_t)1 << 20;
+        fp.desc = st->d_desc;
+        fp.table = f->d_img[var];
+        fp.n_states = f->dfa.n;
+        fp.x = y;
+        fp.k = st->map.k;
+        fp.valid_mask = st->map.valid_mask;
+        for (int s = 0; s < KMAX; s++) {
+            const bool v = (st->map.valid_mask >> s) & 1u;
+            fp.end[s] = v ? to_int(f, st->map.end[s]) : st->map.end[s];
+            fp.count[s] = st->map.count[s];
+        }
+        fp.tail_bits = bits ? (uint32_t)(st->len & 7) : 0u;
+        fp.bittab = f->d_bittab;
+        fp.out = f->d_fix;
+        fp.stats = f->d_stats;
+        fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows,
+                       f->ncls, f->cl_magic, 4, 1u << 28};
+        FixFn fn = get_fix(var);
+        const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
+        CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        fn<<<1, kThreads, smem, f->stream>>>(fp);
+        CK(cudaGetLastError());
+        unsigned long long h[5];
+        CK(cudaMemcpyAsync(h, f->d_fix, sizeof(h), cudaMemcpyDeviceToHost, f->stream));
+        CK(cudaStreamSynchronize(f->stream));
+        if (h[0]) {
+            *end = to_user(f, (uint32_t)h[1]);
+            *count = h[2];
+            return FSM_OK;
+        }
+        y = (uint32_t)h[1];
+        cy = h[2];
+        const uint64_t t = h[4];
+        resume_byte = t * st->tile_bytes > st->head ? std::min<uint64_t>(t * st->tile_bytes - st->head, whole) : 0;
     }
-    fp.out = f->d_fix;
-    fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows,
-                   f->ncls, f->cl_magic, 4, 1u << 28};
-    FixFn fn = get_fix(var);
-    const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
-    CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    fn<<<1, kThreads, smem, f->stream>>>(fp);
-    CK(cudaGetLastError());
-    unsigned long long h[4];
-    CK(cudaMemcpyAsync(h, f->d_fix, sizeof(h), cudaMemcpyDeviceToHost, f->stream));
-    CK(cudaStreamSynchronize(f->stream));
-    if (h[0]) {
-        *end = to_user(f, (uint32_t)h[1]);
-        *count = h[2];
-        return FSM_OK;
-    }
-    // no convergence: exact parallel re-run of the shard from the true start
-    RunSpec r{nullptr, st->input, st->len, st->k, false, 0, to_int(f, true_start), nullptr, f->d_result, var,
-              FSM_MERGE_PARALLEL};
+    // the paths did not meet within the walk's budget: run the rest of the shard from the state
+    // reached with the parallel known-start kernel (exact)
+    const uint64_t rest = st->len - (bits ? resume_byte * 8 : resume_byte);
+    RunSpec r{nullptr, st->input + resume_byte, rest, st->k, false, 0, y, nullptr, f->d_result, var, FSM_MERGE_PARALLEL};
+    r.accumulate = true;
     int rc = launch_run(f, r);
     if (rc) return rc;
     if ((rc = finish_sync(f, f->d_result))) return rc;
     *end = to_user(f, f->h_result->final_state);
-    *count = f->h_result->count;
+    *count = f->h_result->count + cy;
     return FSM_OK;
 }
 
-extern "C" void fsm_shard_free(fsm_shard_t *st) { delete st; }
+extern "C" void fsm_shard_free(fsm_shard_t *st)
+{
+    if (!st) return;
+    cudaFree(st->d_desc);
+    delete st;
+}
 
 // ---------------------------------------------------------------------------- test hooks ----
 extern "C" int fsm_debug_set_spec(fsm_t *f, const uint32_t *sets, uint32_t n_chunks, uint32_t k, uint32_t chunk_bytes)
@@ -1291,6 +1359,15 @@ extern "C" int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *inpu
                 group_of[j] = (int)i;
                 g.push_back(j);
             }
+        if (K > kMultiMaxK) {  // fused multi-FSM kernels exist for K <= 8: one launch per DFA here
+            for (uint32_t j : g) {
+                RunSpec r{nullptr, input, len, k[j], false, 0, fsms[j]->start_int, nullptr, fsms[j]->d_result, -1,
+                          FSM_MERGE_PARALLEL};
+                r.accumulate = true;
+                if ((rc = launch_run(fsms[j], r))) break;
+            }
+            continue;
+        }
         uint32_t T = 0, chunk = 0;
         pick_geometry(fsms[i], len_bytes, K, T, chunk);
         size_t smem = 0;

@@ -17,26 +17,31 @@ typedef void (*MultiFn)(Params, const Params *, uint32_t);
 #define FSM_CAT2(a, b) a##b
 #define FSM_CAT(a, b) FSM_CAT2(a, b)
 
+// Alg. 2 (hash check) kernels exist for the large-k instantiations only (the paper uses the hash
+// form for k > 12); the host falls back to Alg. 1 elsewhere.
 template <int K>
-static KernelFn pick(bool split)
+static KernelFn pick(bool split, bool hash)
 {
+    if constexpr (K >= 12) {
+        if (hash) return speck_kernel<K, FSM_VAR, false, true>;  // Alg. 2 kernels are unsplit
+    }
     if constexpr (split_kernel(FSM_VAR, K)) {
         if (split) return speck_kernel<K, FSM_VAR, true>;
     }
     return speck_kernel<K, FSM_VAR, false>;
 }
 
-KernelFn FSM_CAT(get_kernel_, FSM_VAR_NAME)(int K, bool split)
+KernelFn FSM_CAT(get_kernel_, FSM_VAR_NAME)(int K, bool split, bool hash)
 {
     switch (K) {
-    case 1: return pick<1>(split);
-    case 2: return pick<2>(split);
-    case 3: return pick<3>(split);
-    case 4: return pick<4>(split);
-    case 6: return pick<6>(split);
-    case 8: return pick<8>(split);
-    case 12: return pick<12>(split);
-    default: return pick<16>(split);
+    case 1: return pick<1>(split, false);
+    case 2: return pick<2>(split, false);
+    case 3: return pick<3>(split, false);
+    case 4: return pick<4>(split, false);
+    case 6: return pick<6>(split, false);
+    case 8: return pick<8>(split, false);
+    case 12: return pick<12>(split, hash);
+    default: return pick<16>(split, hash);
     }
 }
 
@@ -49,8 +54,7 @@ MultiFn FSM_CAT(get_multi_, FSM_VAR_NAME)(int K)
     case 4: return speck_multi_kernel<4, FSM_VAR>;
     case 6: return speck_multi_kernel<6, FSM_VAR>;
     case 8: return speck_multi_kernel<8, FSM_VAR>;
-    case 12: return speck_multi_kernel<12, FSM_VAR>;
-    default: return speck_multi_kernel<16, FSM_VAR>;
+    default: return nullptr;  // K >= 12: the host runs those DFAs one launch each
     }
 }
 

@@ -114,7 +114,8 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
                 uint32_t cx = 0, cyc = 0;
                 int conv = -1;
                 uint64_t pos = b;
-                while (conv < 0 && pos < e) {
+                const uint64_t wend = min(e, b + kLockstepWindow);
+                while (conv < 0 && pos < wend) {
                     const typename TB::Row r = tb.row(__ldg(p.in + pos));
                     x = tb.apply(r, x, cx);
 #pragma unroll
@@ -127,6 +128,7 @@ __global__ void __launch_bounds__(kThreads) seq_walk_kernel(Params p, SeqBuf sb)
                         }
                     pos++;
                 }
+                for (; conv < 0 && pos < e; pos++) x = tb.apply(tb.row(__ldg(p.in + pos)), x, cx);  // alone
                 reexec++;
                 rebytes += pos - b;
                 chain++;  // consecutive re-executed chunks (reset by a speculated hit)

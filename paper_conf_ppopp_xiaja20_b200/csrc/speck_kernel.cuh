@@ -34,6 +34,11 @@ constexpr int kThreads = 256;  // auxiliary kernels
 constexpr int kExt = 4;
 constexpr uint32_t kExtWindow = 128;  // bytes of lockstep per chunk; |count delta| <= 8 * 128 fits 12 bits
 constexpr uint32_t kExtNone = 0xFFFFu;
+constexpr uint32_t kHashSize = 32;
+// Early-exit re-execution (R3) runs the chunk's chains in lockstep for at most this many bytes; past
+// it (paths that do not meet, e.g. permutation DFAs with k < N) the re-executed path continues alone:
+// K + 1 lookups per byte only where a meeting is likely, one afterwards.  Exact either way.
+constexpr uint32_t kLockstepWindow = 256;  // Alg. 2 buckets per thread (reading A10: next power of two >= 2k, k <= 16)
 // Threads per tile (one chunk per thread) of the fused kernel, by the number of chains K: large
 // CTAs keep few tiles in flight (short look-back windows) at one CTA per SM; the register budget
 // caps them for large K.
@@ -837,6 +842,86 @@ __device__ __forceinline__ void compose(uint32_t (&eob)[K], uint32_t (&cnt)[K], 
     }
 }
 
+// Alg. 2: the hash implementation of the runtime check, which the paper uses for large
+// k (k > 12, footnote P:200) because Alg. 1 costs O(k^2).  B200 form: instead of dynamically
+// indexed per-thread arrays (which the paper notes spill to local memory), every thread owns
+// one column of a shared-memory table -- word (row * T + tid), so a warp's accesses are conflict-free:
+//   rows 0 .. kHashSize-1   hash_init_states: bucket h holds (slot << 16 | start), open addressing
+//                           (linear probing) in place of fixed-capacity chains; HASH_SIZE = 32 = the
+//                           next power of two >= 2k for 8 < k <= 16 and hash = s mod HASH_SIZE (A10)
+//   rows 32 .. 32+K-1       hash_end_states of the thread's current mapping (eob per slot)
+//   rows 32+K .. 32+2K-1    its counts
+// Step 1 (lines 7-12) is built once per scan from the thread's own start set (a lane's mapping is
+// always keyed on its own first chunk's starts); before each scan level the lane publishes its
+// current ends and counts, and step 2 (lines 14-28) probes the RIGHT lane's column: O(k) per slot
+// set, no shuffles of the right mapping and no k x k compare network.  Results are identical to
+// Alg. 1 (the same matches; starts are distinct, reading A6).
+constexpr uint32_t kHashEmpty = 0xFFFFFFFFu;
+template <int K>
+__device__ __forceinline__ void hash_build(uint32_t *hs, uint32_t T, uint32_t tid, const uint32_t (&S)[K])
+{
+#pragma unroll
+    for (uint32_t h = 0; h < kHashSize; h++) hs[h * T + tid] = kHashEmpty;
+#pragma unroll
+    for (int j = 0; j < K; j++)
+        if (S[j] != NOSTATE) {
+            uint32_t h = S[j] & (kHashSize - 1);
+            while (hs[h * T + tid] != kHashEmpty) h = (h + 1) & (kHashSize - 1);
+            hs[h * T + tid] = ((uint32_t)j << 16) | S[j];
+        }
+}
+template <int K>
+__device__ __forceinline__ void hash_publish(uint32_t *hs, uint32_t T, uint32_t tid, const uint32_t (&eob)[K],
+                                             const uint32_t (&cnt)[K])
+{
+#pragma unroll
+    for (int s = 0; s < K; s++) {
+        hs[(kHashSize + s) * T + tid] = eob[s];
+        hs[(kHashSize + K + s) * T + tid] = cnt[s];
+    }
+}
+// (L x R)[s] with R published in column rt (Alg. 2 step 2); same semantics as compose().
+template <int K>
+__device__ __forceinline__ void compose_hash(uint32_t (&eob)[K], uint32_t (&cnt)[K], const uint32_t *hs, uint32_t T,
+                                             uint32_t rt, uint32_t first_r, const uint32_t *ext)
+{
+#pragma unroll
+    for (int s = 0; s < K; s++) {
+        const uint32_t x = eob[s];
+        if ((x >> 16) == COMPLETE) {
+            const uint32_t st = x & 0xFFFFu;
+            uint32_t h = st & (kHashSize - 1), j = 0xFFFFFFFFu;
+            for (;;) {  // at most K occupied buckets of 2K: terminates at an empty one
+                const uint32_t e = hs[h * T + rt];
+                if (e == kHashEmpty) break;
+                if ((e & 0xFFFFu) == st) {
+                    j = e >> 16;
+                    break;
+                }
+                h = (h + 1) & (kHashSize - 1);
+            }
+            uint32_t ne = st | (first_r << 16), nc = 0;
+            if (j != 0xFFFFFFFFu) {
+                ne = hs[(kHashSize + j) * T + rt];
+                nc = hs[(kHashSize + K + j) * T + rt];
+            } else if (ext) {
+                const uint32_t *ex = ext + first_r * kExt;
+#pragma unroll
+                for (int q = 0; q < kExt; q++) {
+                    const uint32_t v = ex[q];
+                    if ((v & 0xFFFFu) == st) {
+                        const uint32_t l = (v >> 16) & 0xFu;
+                        ne = hs[(kHashSize + l) * T + rt];
+                        nc = hs[(kHashSize + K + l) * T + rt] + (uint32_t)((int32_t)v >> 20);
+                    }
+                }
+            }
+            eob[s] = ne;
+            cnt[s] += nc;
+        }
+    }
+}
+
 // Test hook (fsm_debug_get_merge): the lane's mapping after scan level `level` (0 = the chunk's own).
 template <int K>
 __device__ __forceinline__ void dbg_record(uint4 *dbg, int level, const uint32_t (&S)[K], const uint32_t (&eob)[K],
@@ -852,13 +937,27 @@ __device__ __forceinline__ void dbg_record(uint4 *dbg, int level, const uint32_t
 // chunk distance between lanes.  Level d composes lane i with lane i + d, so lane 0 after d = 1 is
 // M_0 x M_1, lane 2 is M_2 x M_3, and lane 0 after d = 2 is (M_0 x M_1) x (M_2 x M_3): the merge tree
 // of Fig. 4b.  dbg (test hook, normally null) records every level.
-template <int K>
+template <int K, bool HASH = false>
 __device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eob)[K], uint32_t (&cnt)[K], bool &ident,
                                                  uint32_t first0, uint32_t step, const uint32_t *ext = nullptr,
-                                                 uint4 *dbg = nullptr)
+                                                 uint4 *dbg = nullptr, uint32_t *hs = nullptr)
 {
     const int lane = threadIdx.x & 31;
     if (dbg) dbg_record<K>(dbg, 0, S, eob, cnt, ident);
+    if constexpr (HASH) {
+        const uint32_t T = blockDim.x, tid = threadIdx.x;
+        hash_build<K>(hs, T, tid, S);
+#pragma unroll
+        for (int d = 1, level = 1; d < 32; d <<= 1, level++) {
+            const bool ir = __shfl_down_sync(0xFFFFFFFFu, (int)ident, d) != 0;
+            hash_publish<K>(hs, T, tid, eob, cnt);
+            __syncwarp();
+            if (lane + d < 32 && !ir && !ident) compose_hash<K>(eob, cnt, hs, T, tid + d, first0 + (lane + d) * step, ext);
+            __syncwarp();
+            if (dbg) dbg_record<K>(dbg, level, S, eob, cnt, ident);
+        }
+        return;
+    }
 #pragma unroll
     for (int d = 1, level = 1; d < 32; d <<= 1, level++) {
         uint32_t Sr[K], er[K], cr[K];
@@ -879,10 +978,13 @@ __device__ __forceinline__ void warp_suffix_scan(uint32_t (&S)[K], uint32_t (&eo
 // double-buffered -- buffer b at offset b * buf -- and there is no stash (re-execution and eager
 // completion read the chunk's first bytes from L2 instead).
 struct Layout {
-    uint32_t qe, qc, sj, ws, we, wc, wi, misc, stash, ext, total, buf;
-    __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t start, bool split = false)
+    uint32_t qe, qc, sj, ws, we, wc, wi, misc, stash, ext, hs, total, buf;
+    __host__ __device__ Layout(uint32_t T, uint32_t K, uint32_t start, bool split = false, bool hash = false)
     {
         uint32_t o = start;
+        // Alg. 2 scratch: one column per thread of kHashSize buckets + K end states + K counts
+        hs = o;
+        if (hash) o += T * (kHashSize + 2 * K) * 4;
         qe = o;  o += T * K * 4;
         qc = o;  o += T * K * 4;
         sj = o;  o += T * K * 2;
@@ -1010,6 +1112,7 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
         uint32_t cx = 0, cyc = 0;
         int conv = -1;
         uint64_t pos = b;
+        const uint64_t wend = min(e, b + kLockstepWindow);
         auto one = [&](uint32_t byte) {
             const typename TB::Row r = tb.row(byte);
             st = tb.apply(r, st, cx);
@@ -1032,11 +1135,11 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
             }
         }
         if (t.aligned) {
-            while (conv < 0 && (pos & 15) && pos < e) {
+            while (conv < 0 && (pos & 15) && pos < wend) {
                 one(__ldg(t.in + pos));
                 pos++;
             }
-            while (conv < 0 && pos + 16 <= e) {
+            while (conv < 0 && pos + 16 <= wend) {
                 const uint4 v = ldg128(t.in + pos);
                 uint32_t used = 0;
 #pragma unroll 1
@@ -1048,9 +1151,21 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
                 pos += used;
             }
         }
-        while (conv < 0 && pos < e) {
+        while (conv < 0 && pos < wend) {
             one(__ldg(t.in + pos));
             pos++;
+        }
+        if (conv < 0 && pos < e) {  // past the lockstep window: the re-executed path alone
+            if (t.aligned) {
+                for (; (pos & 15) && pos < e; pos++) st = tb.apply(tb.row(__ldg(t.in + pos)), st, cx);
+                for (; pos + 16 <= e; pos += 16) {
+                    const uint4 v = ldg128(t.in + pos);
+                    const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                    for (int q = 0; q < 16; q++) st = tb.apply(tb.row((w4[q >> 2] >> (8 * (q & 3))) & 0xFFu), st, cx);
+                }
+            }
+            for (; pos < e; pos++) st = tb.apply(tb.row(__ldg(t.in + pos)), st, cx);
         }
         chain = c == last_c + 1 ? chain + 1 : 1;
         last_c = c;
@@ -1108,11 +1223,11 @@ __device__ __forceinline__ void add_stats(DevStats *S, const ReCount &rc, bool t
 // slots (R5, the top p.preresolve tile-start candidates), publication of A, decoupled look-back,
 // own inclusive prefix P (resolving the true path's broken slot if it was left unresolved), and the
 // result.
-template <int K, class TB>
+template <int K, bool HASH, class TB>
 __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uint32_t tile, uint64_t tile_base,
                                               uint32_t nch_max, uint32_t *Qe, uint32_t *Qc, const uint16_t *Sj,
                                               const uint32_t *stash, const uint32_t *Ext, uint32_t start_state,
-                                              unsigned long long start_count, uint32_t ksel)
+                                              unsigned long long start_count, uint32_t ksel, uint32_t *hs)
 {
     const int lane = threadIdx.x & 31;
     TileCtx t;
@@ -1242,7 +1357,7 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
 #pragma unroll
             for (int l = 0; l < K; l++) S2[l] = NOSTATE, e2[l] = ABSENT << 16, c2[l] = 0;
         }
-        warp_suffix_scan<K>(S2, e2, c2, id2, 0, 1);
+        warp_suffix_scan<K, HASH>(S2, e2, c2, id2, 0, 1, nullptr, nullptr, hs);
         int brk = 32;
         {
             uint32_t ne = 0, nc = 0;
@@ -1385,10 +1500,11 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
 // other warps (T - 32 chunks per tile) hand each tile's state over in one of two buffers and go
 // straight on to the next tile, so the serial epilogue (pre-resolution re-executions, look-back)
 // overlaps the next tile's local phase instead of idling the SM at a barrier.
-template <int K, int VAR, bool MULTI, bool SPLIT = false>
+template <int K, int VAR, bool MULTI, bool SPLIT = false, bool HASH = false>
 __device__ __forceinline__ void speck_body(const Params &p0, const Params *__restrict__ pm, uint32_t M)
 {
     static_assert(!(MULTI && SPLIT), "multi-FSM runs use the unsplit body");
+    static_assert(!HASH || K > 8, "Alg. 2 is instantiated for large k only (P:200)");
     using TB = typename TableFor<VAR>::type;
     extern __shared__ __align__(16) uint8_t smem[];  // no static shared memory: see kSmemWindowBase
 
@@ -1398,7 +1514,8 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
     const uint32_t j = threadIdx.x;
 
     // MULTI: p0.table_bytes is the group's largest table image, so one layout serves every DFA
-    const Layout L(T, K, scratch_offset(VAR, p0.table_bytes), SPLIT);
+    const Layout L(T, K, scratch_offset(VAR, p0.table_bytes), SPLIT, HASH);
+    uint32_t *const hs = reinterpret_cast<uint32_t *>(smem + L.hs);  // Alg. 2 columns (HASH only)
     check_smem_window(VAR, L.total);
     TB tb;
     if (!MULTI) tb.setup(smem, p0.table, p0.n_states, kconst(p0));
@@ -1428,10 +1545,10 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
             const uint32_t tile = s_tiles[bb];
             if (tile >= p0.ntiles) break;
             const uint32_t o = bb * L.buf;
-            tile_epilogue<K>(tb, p0, tile, (uint64_t)tile * TW * p0.chunk, TW,
-                             reinterpret_cast<uint32_t *>(smem + L.qe + o), reinterpret_cast<uint32_t *>(smem + L.qc + o),
-                             reinterpret_cast<const uint16_t *>(smem + L.sj + o), nullptr,
-                             reinterpret_cast<const uint32_t *>(smem + L.ext + o), start_state, start_count, p0.k);
+            tile_epilogue<K, HASH>(tb, p0, tile, (uint64_t)tile * TW * p0.chunk, TW,
+                                   reinterpret_cast<uint32_t *>(smem + L.qe + o), reinterpret_cast<uint32_t *>(smem + L.qc + o),
+                                   reinterpret_cast<const uint16_t *>(smem + L.sj + o), nullptr,
+                                   reinterpret_cast<const uint32_t *>(smem + L.ext + o), start_state, start_count, p0.k, hs);
             __syncwarp();
             named_arrive(4 + bb, T);
         }
@@ -1568,8 +1685,8 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
 #endif
         // ---- a5: warp stage (chunks warp*32 .. warp*32+31)
         __syncwarp();  // the lanes' eager-completion entries are read by the scan
-        warp_suffix_scan<K>(S, eob, cnt, ident, (uint32_t)warp * 32, 1, Ext,
-                            (p.dbg && tile == 0 && warp == 0) ? p.dbg : nullptr);
+        warp_suffix_scan<K, HASH>(S, eob, cnt, ident, (uint32_t)warp * 32, 1, Ext,
+                                  (p.dbg && tile == 0 && warp == 0) ? p.dbg : nullptr, hs);
 
         // ---- a6: block stage
         if (lane == 0) {
@@ -1597,7 +1714,7 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
 #pragma unroll
                 for (int s = 0; s < K; s++) S2[s] = NOSTATE, e2[s] = ABSENT << 16, c2[s] = 0;
             }
-            warp_suffix_scan<K>(S2, e2, c2, id2, 0, 32, Ext);
+            warp_suffix_scan<K, HASH>(S2, e2, c2, id2, 0, 32, Ext, nullptr, hs);
             __syncwarp();
             if (lane < W) {
 #pragma unroll
@@ -1637,16 +1754,16 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
         if (warp != 0) continue;
 
         // ================= warp 0: tile epilogue (pre-resolution, look-back, publication) =====
-        tile_epilogue<K>(tb, p, tile, tile_base, TW, Qe, Qc, Sj, reinterpret_cast<const uint32_t *>(smem + L.stash), Ext,
-                         start_state, start_count, ksel);
+        tile_epilogue<K, HASH>(tb, p, tile, tile_base, TW, Qe, Qc, Sj, reinterpret_cast<const uint32_t *>(smem + L.stash),
+                               Ext, start_state, start_count, ksel, hs);
     }
 }
 
 // SPLIT is chosen per launch by the host: split_kernel(VAR, K) and the double-buffered layout fits.
-template <int K, int VAR, bool SPLIT>
+template <int K, int VAR, bool SPLIT, bool HASH = false>
 __global__ void __launch_bounds__(max_threads(K), min_blocks(K)) speck_kernel(Params p)
 {
-    speck_body<K, VAR, false, SPLIT>(p, nullptr, 1);
+    speck_body<K, VAR, false, SPLIT, HASH>(p, nullptr, 1);
 }
 
 template <int K, int VAR>

@@ -23,6 +23,7 @@ VARIANT_NAMES = {0: "P4", 1: "P8", 2: "B", 3: "G", 5: "HS", 6: "CL", 7: "N8", 8:
 FSM_MERGE_PARALLEL, FSM_MERGE_SEQUENTIAL = 0, 1
 FSM_EAGER_OFF = 1
 FSM_PRERESOLVE_NONE = 0x80000000
+FSM_CHECK_AUTO, FSM_CHECK_NESTED, FSM_CHECK_HASH = 0, 1, 2
 
 # every symbol declared in include/fsmspec.h
 EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_set_stream",
@@ -36,7 +37,7 @@ class fsm_options(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
                 ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32),
                 ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32), ("preresolve", ctypes.c_uint32),
-                ("grid_sms", ctypes.c_uint32)]
+                ("grid_sms", ctypes.c_uint32), ("check", ctypes.c_uint32)]
 
 
 class fsm_tuning(ctypes.Structure):
@@ -53,7 +54,7 @@ class fsm_stats(ctypes.Structure):
                 ("eager_resolved", ctypes.c_uint64), ("max_miss_chain", ctypes.c_uint64),
                 ("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
                 ("variant", ctypes.c_uint32), ("k_slots", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32),
-                ("preresolve", ctypes.c_uint32)]
+                ("preresolve", ctypes.c_uint32), ("check", ctypes.c_uint32)]
 
 
 class fsm_shard_map(ctypes.Structure):
@@ -228,9 +229,9 @@ class FSM:
 
     def set_options(self, chunk_bytes: int = 0, threads_per_tile: int = 0, variant: int = FSM_VARIANT_AUTO,
                     merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0, lookback_len: int = 0,
-                    eager_window: int = 0, preresolve: int = 0, grid_sms: int = 0) -> None:
+                    eager_window: int = 0, preresolve: int = 0, grid_sms: int = 0, check: int = 0) -> None:
         o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm, lookback_len, eager_window,
-                        preresolve, grid_sms)
+                        preresolve, grid_sms, check)
         _check(lib().fsm_set_options(self._h, ctypes.byref(o)), "fsm_set_options")
 
     def options(self) -> dict:

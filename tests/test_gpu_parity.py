@@ -319,6 +319,55 @@ def test_shard_maps_compose_and_fixup(G, k):
         assert (x, total) == exp
 
 
+@pytest.mark.parametrize("kind", ["rand16_6", "html", "div7", "rand8_8_unaligned"])
+def test_shard_fixup_walks_tile_descriptors(kind):
+    """SURVEY.md 8.e fix-up: for every true start that the shard did not speculate (k < |image(halo)|),
+    fsm_shard_fixup equals the oracle from that start.  For converging DFAs the walk re-executes
+    at most one tile (it joins a shard slot's path at the first tile boundary) and costs < 1 % of the
+    shard run; for a permutation DFA (Div7, paths never meet) it falls back to the parallel kernel."""
+    off = 0
+    if kind == "html":
+        d, data, k, nsym = dfas.html_tokenizer(), streams.html_bytes(64 << 20, 9), 1, None
+    elif kind == "div7":
+        d, k = dfas.div7(), 2
+        data = streams.random_bits(8 * (16 << 20), 6)
+        nsym = 8 * (16 << 20)
+    else:
+        n, m = int(kind.split("_")[0][4:]), int(kind.split("_")[1])
+        d, data, k, nsym = dfas.random_dfa(n, m, seed=n * m), streams.splitmix_bytes(n + m, 0, 64 << 20), 2, None
+        if "unaligned" in kind:
+            off = 5
+    nbytes = data.size
+    lo = (nbytes // 3) // 32 * 32 + off
+    buf, base = dev(data)
+    shard = data[lo:]
+    with FSM.from_dfa(d) as f:
+        s_sym = (nbytes - lo) * 8 if d.bit_mode else nbytes - lo
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record()
+        m, st = f.run_shard(base + lo, s_sym, halo=base + lo - 1, halo_len=1, k=k, keep=True)
+        t1.record()
+        torch.cuda.synchronize()
+        shard_ms = t0.elapsed_time(t1)
+        spec = {s for s, _, _ in m.slots()}
+        n_int = d.n_states
+        misses = [x for x in range(n_int) if x not in spec]
+        assert misses, "k < |image(halo)| needed"
+        for x in misses[:6]:
+            exp = seq.run_from(d, x, shard, s_sym if d.bit_mode else None)
+            t0.record()
+            got = f.shard_fixup(st, x)
+            t1.record()
+            torch.cuda.synchronize()
+            assert got == exp, (kind, x)
+            fst = f.stats()
+            if kind != "div7":
+                assert fst["reexec_true"] <= 1, fst          # touched at most one tile
+                assert t0.elapsed_time(t1) < 0.01 * shard_ms + 0.5, (t0.elapsed_time(t1), shard_ms)
+        st.close()
+
+
 # --------------------------------------------------------------------- look-back windows (R7)
 def _wl_cases():
     pats = dfas.snort_patterns(300, seed=8)

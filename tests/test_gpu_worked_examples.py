@@ -200,3 +200,57 @@ def test_unaligned_input_peels_one_sector():
                 f.set_options(lookback_len=lb)
                 for k in (1, 2):
                     assert f.run_spec_k(buf.data_ptr() + off, data.size, k) == exp, (off, lb, k)
+
+
+# --------------------------------------------------------------------- Alg. 2 (hash check) on the GPU
+@pytest.mark.parametrize("n,m", [(16, 12), (40, 16), (255, 14)])
+@pytest.mark.parametrize("k", [12, 13, 16])
+def test_hash_check_matches_nested(n, m, k):
+    """Alg. 2 and Alg. 1 give identical results and identical re-execution
+    counts for every variant that has the hash form; the run reports which check it used."""
+    if k > n:
+        pytest.skip("k <= N")
+    d = dfas.random_dfa(n, m, seed=500 + n + m)
+    data = streams.splitmix_bytes(600 + n, 0, (3 << 20) + 11)
+    exp = seq.run(d, data)
+    for var in ("B", "G", "R16", "CL", "HS"):
+        if var == "R16" and n > 16:
+            continue
+        with FSM.from_dfa(d) as f:
+            buf, ptr = dev(data)
+            stats = {}
+            for chk in (fsmspec.FSM_CHECK_NESTED, fsmspec.FSM_CHECK_HASH):
+                try:
+                    f.set_options(variant=VARIANTS[var], check=chk, chunk_bytes=512,
+                                  eager_window=fsmspec.FSM_EAGER_OFF)
+                except fsmspec.FsmError:
+                    break  # the DFA does not fit this variant
+                assert f.run_spec_k(ptr, data.size, k) == exp, (var, chk)
+                stats[chk] = f.stats()
+            if len(stats) == 2:
+                a, b = stats[fsmspec.FSM_CHECK_NESTED], stats[fsmspec.FSM_CHECK_HASH]
+                assert a["check"] == fsmspec.FSM_CHECK_NESTED
+                if b["check"] == fsmspec.FSM_CHECK_HASH:
+                    # the chunk-level true-path miss count does not depend on the tile geometry
+                    assert a["reexec_true"] == b["reexec_true"], (var, a, b)
+
+
+def test_hash_check_merge_tree_identical():
+    """With injected 12-slot sets on tiny chunks, every level of the warp merge tree read back
+    from the GPU is the same under Alg. 1 and Alg. 2 (including invalid slots and where they broke)."""
+    d = dfas.random_dfa(16, 14, seed=9)
+    rng = np.random.default_rng(4)
+    data = rng.integers(0, 256, 64).astype(np.uint8)
+    sets = [list(rng.choice(16, 12, replace=False)) for _ in range(32)]
+    out = {}
+    for chk in (fsmspec.FSM_CHECK_NESTED, fsmspec.FSM_CHECK_HASH):
+        with FSM.from_dfa(d) as f:
+            f.set_options(variant=VARIANTS["G"], check=chk)
+            f.debug_set_spec(sets, chunk_bytes=2)
+            buf, ptr = dev(data)
+            assert f.run_spec_k(ptr, data.size, 12) == seq.run(d, data)
+            assert f.stats()["check"] == chk
+            m = f.debug_get_merge()
+            out[chk] = [[m.mapping(lv, lane) for lane in range(32)] for lv in range(6)]
+            out[chk].append([[int(m.brk[lv][lane][s]) for s in range(16)] for lv in range(6) for lane in range(32)])
+    assert out[fsmspec.FSM_CHECK_NESTED] == out[fsmspec.FSM_CHECK_HASH]

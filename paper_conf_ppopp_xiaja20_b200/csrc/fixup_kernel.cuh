@@ -35,6 +35,7 @@ struct FixParams {
     uint32_t n_states;
     uint32_t x;                // true start (internal id)
     uint32_t k;                // shard slots
+    uint32_t kslots;           // aggregate slots per descriptor (the keyed run's instantiated K)
     uint32_t valid_mask;
     uint32_t end[KMAX];        // shard map (internal ids) and counts
     unsigned long long count[KMAX];
@@ -85,8 +86,8 @@ __global__ void __launch_bounds__(kThreads) fixup_kernel(FixParams f)
         }
         // (2) pass through the tile with a complete aggregate slot
         uint4 a = make_uint4(NOSTATE, 0u, 0u, 1u);
-        if (lane < KMAX) a = D.aslot[lane];
-        const bool have = lane < (int)KMAX && a.x != NOSTATE;
+        if ((uint32_t)lane < f.kslots) a = D.aslot[lane];  // slots >= K of a descriptor are stale
+        const bool have = (uint32_t)lane < f.kslots && a.x != NOSTATE;
         const unsigned hm = __ballot_sync(0xFFFFFFFFu, have && a.w == 0u && a.x == y);
         if (hm) {
             const int l = __ffs(hm) - 1;

@@ -193,7 +193,7 @@ struct fsm_shard {
     fsm_shard_map map{};
     // keyed runs: the tile descriptors (aggregates A_t, prefixes P_t) the fix-up walks
     TileDesc *d_desc = nullptr;
-    uint32_t ntiles = 0, head = 0;
+    uint32_t ntiles = 0, head = 0, kslots = 0;
     uint64_t tile_bytes = 0;
 };
 
@@ -532,9 +532,9 @@ static int variant_of(const fsm *f, int force, uint32_t k = 1)
 // Geometry: T chunks per tile (CTA threads), chunk bytes.  Large inputs: the largest CTA the
 // register budget allows for K and 4 KiB chunks.  Small inputs: shrink the CTA, then the chunk,
 // so that every SM still gets a few tiles.
-static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, uint32_t &T, uint32_t &chunk)
+static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, int var, uint32_t &T, uint32_t &chunk)
 {
-    const uint32_t tmax = (uint32_t)max_threads(K);
+    const uint32_t tmax = (uint32_t)max_threads(K, var);
     T = f->opt.threads_per_tile ? std::min<uint32_t>(f->opt.threads_per_tile, tmax) : tmax;
     if (!f->opt.threads_per_tile)
         while (T > 128 && len_bytes < (uint64_t)f->num_sms * T * 4096) T >>= 1;
@@ -608,7 +608,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     }
     const uint64_t len_bytes = ulen_bytes + head;  // kernel coordinates
     uint32_t T = 0, chunk = 0;
-    pick_geometry(f, r.geom_len_bytes ? std::max(r.geom_len_bytes, ulen_bytes) : ulen_bytes, K, T, chunk);
+    pick_geometry(f, r.geom_len_bytes ? std::max(r.geom_len_bytes, ulen_bytes) : ulen_bytes, K, var, T, chunk);
     if (r.force_T) T = r.force_T;
     if (r.force_chunk) chunk = r.force_chunk;
     const bool dbg = f->dbg_chunk != 0 && !r.multi;
@@ -975,6 +975,7 @@ extern "C" int fsm_run_shard(fsm_t *f, const uint8_t *input, uint64_t len, const
             st->ntiles = (uint32_t)f->last.tiles;
             st->tile_bytes = (uint64_t)f->last.threads_per_tile * f->last.chunk_bytes;
             st->head = f->last_head;
+            st->kslots = f->last.k_slots;
             if (cudaMalloc(&st->d_desc, st->ntiles * sizeof(TileDesc)) != cudaSuccess ||
                 cudaMemcpyAsync(st->d_desc, f->d_desc, st->ntiles * sizeof(TileDesc), cudaMemcpyDeviceToDevice,
                                 f->stream) != cudaSuccess ||
@@ -1017,6 +1018,7 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         fp.n_states = f->dfa.n;
         fp.x = y;
         fp.k = st->map.k;
+        fp.kslots = st->kslots;
         fp.valid_mask = st->map.valid_mask;
         for (int s = 0; s < KMAX; s++) {
             const bool v = (st->map.valid_mask >> s) & 1u;
@@ -1369,7 +1371,7 @@ extern "C" int fsm_run_multi(fsm_t *const *fsms, uint32_t m, const uint8_t *inpu
             continue;
         }
         uint32_t T = 0, chunk = 0;
-        pick_geometry(fsms[i], len_bytes, K, T, chunk);
+        pick_geometry(fsms[i], len_bytes, K, var, T, chunk);
         size_t smem = 0;
         uint32_t tbytes = 0;
         for (uint32_t n = 0; n < g.size() && rc == FSM_OK; n++) {

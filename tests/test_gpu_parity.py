@@ -319,7 +319,7 @@ def test_shard_maps_compose_and_fixup(G, k):
         assert (x, total) == exp
 
 
-@pytest.mark.parametrize("kind", ["rand16_6", "html", "div7", "rand8_8_unaligned"])
+@pytest.mark.parametrize("kind", ["rand16_6", "html", "div7", "rand8_3_unaligned"])
 def test_shard_fixup_walks_tile_descriptors(kind):
     """SURVEY.md 8.e fix-up: for every true start that the shard did not speculate (k < |image(halo)|),
     fsm_shard_fixup equals the oracle from that start.  For converging DFAs the walk re-executes
@@ -535,3 +535,31 @@ def test_html_cl_large_k(k):
     for lb in (0, 64):
         got, st = gpu_run(d, data, k=k, variant=VARIANTS["CL"], lookback_len=lb)
         assert got == exp, (k, lb, st)
+
+
+# --------------------------------------------------------------------- production geometry
+FULL_CASES = [("P4", 4, 2), ("N8", 8, 2), ("P8", 8, 3), ("R16", 16, 2), ("B", 64, 4), ("G", 1000, 3),
+              ("HS", 3000, 3), ("CL", 0, 0)]
+
+
+@pytest.mark.parametrize("var,n,m", FULL_CASES)
+def test_full_geometry_parity(var, n, m):
+    """Every table variant at the bench's launch geometry (inputs large enough that pick_geometry
+    chooses the maximal tile and 4 KiB chunks, split kernels where the policy splits) against the
+    oracle, k = 1 and 2, with the default look-back and eager completion."""
+    L = 640 << 20
+    if var == "CL":
+        d = dfas.html_tokenizer()
+        data = streams.html_bytes(L, 21)
+    else:
+        d = dfas.random_dfa(n, m, seed=900 + n)
+        data = streams.splitmix_bytes(31 + n, 0, L)
+    exp = seq.run(d, data)
+    buf, ptr = dev(data)
+    with FSM.from_dfa(d) as f:
+        for k in (1, 2):
+            f.set_options(variant=VARIANTS[var], lookback_len=64 if var == "CL" else 0)
+            assert f.run_spec_k(ptr, L, k) == exp, (var, k)
+            st = f.stats()
+            assert st["chunk_bytes"] == 4096 and st["threads_per_tile"] >= 224, st
+            assert st["variant"] == VARIANTS[var]

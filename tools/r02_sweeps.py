@@ -119,7 +119,10 @@ def sweep_check(out, gib):
             ref = None
 
 
-def sweep_grid(out, gib):
+def sweep_grid(out, gib, scaled=False):
+    """scaled=False: the library's fixed 4 KiB chunks at every grid size.  scaled=True: the number
+    of chunks grows with the grid like the paper's one-chunk-per-thread kernel (chunk bytes =
+    2048 x 148 / SMs), so the sequential merge walks more chunks on bigger grids (Figs. 7-11)."""
     for cfg, ks in (("c4", (1, 4)), ("c2", (4,))):
         d, data, nsym, lb = workload(cfg, gib)
         nbytes = nsym // 8 if d.bit_mode else nsym
@@ -129,12 +132,14 @@ def sweep_grid(out, gib):
                 ref = None
                 for sms in (37, 74, 148):
                     row = {}
+                    chunk = 2048 * 148 // sms if scaled else 0
                     for merge, name in ((fsmspec.FSM_MERGE_PARALLEL, "parallel"), (fsmspec.FSM_MERGE_SEQUENTIAL, "sequential")):
-                        f.set_options(lookback_len=lb, merge=merge, grid_sms=sms)
+                        f.set_options(lookback_len=lb, merge=merge, grid_sms=sms, chunk_bytes=chunk)
                         t, got, st = timed(f, buf.data_ptr(), nsym, k, reps=3)
                         ref = ref or got
                         row[name] = (round(nbytes / t / 1e9, 1), got == ref)
-                    emit(out, sweep="grid", config=cfg, gib=gib, k=k, sms=sms, parallel_gbs=row["parallel"][0],
+                    emit(out, sweep="grid_scaled" if scaled else "grid", config=cfg, gib=gib, k=k, sms=sms,
+                         chunk_bytes=st["chunk_bytes"], parallel_gbs=row["parallel"][0],
                          sequential_gbs=row["sequential"][0], ratio=round(row["parallel"][0] / row["sequential"][0], 2),
                          ok=row["parallel"][1] and row["sequential"][1],
                          paper_v100="parallel/sequential 2.02-6.74x best vs best (P:11); Huffman 289.72/355.32/407.23 vs "
@@ -143,13 +148,14 @@ def sweep_grid(out, gib):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--sweep", required=True, choices=["r5", "check", "grid"])
+    ap.add_argument("--sweep", required=True, choices=["r5", "check", "grid", "grid_scaled"])
     ap.add_argument("--gib", type=float, default=1.0)
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweeps.jsonl"))
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
     with open(a.out, "a") as out:
-        {"r5": sweep_r5, "check": sweep_check, "grid": sweep_grid}[a.sweep](out, a.gib)
+        {"r5": sweep_r5, "check": sweep_check, "grid": sweep_grid,
+         "grid_scaled": lambda o, g: sweep_grid(o, g, True)}[a.sweep](out, a.gib)
 
 
 if __name__ == "__main__":

@@ -40,7 +40,7 @@ __global__ void __launch_bounds__(kThreads) seq_local_kernel(Params p, SeqBuf sb
             acc[s] = 0;
             accf[s] = 0;
         }
-        if (e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf, nullptr, p.lb);
+        if (e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf);
 #pragma unroll
         for (int s = 0; s < K; s++) {
             sb.S[g * K + s] = (uint16_t)(S[s] == NOSTATE ? 0xFFFFu : S[s]);

@@ -44,13 +44,7 @@ constexpr uint32_t kLockstepWindow = 256;  // Alg. 2 buckets per thread (reading
 // caps them for large K.
 // (K = 2, 3 at 768 threads get 85 registers: the multi-chain prologue spills at 64; measured
 // +6 % over 1024 threads for (8, 2, k=2).)
-// K = 1 on the latency-bound variants (CL, B, G, HS) runs two chains per thread (two halves, see
-// local_phase_halves); 768 threads leave it 80 registers, where 1024 threads spilled the hot loop.
-__host__ __device__ constexpr bool two_halves_var(int var) { return var == 6 || var == 2 || var == 3 || var == 5; }
-__host__ __device__ constexpr int max_threads(int K, int var = -1)
-{
-    return K == 1 ? (two_halves_var(var) ? 768 : 1024) : K <= 3 ? 768 : K <= 6 ? 512 : 256;
-}
+__host__ __device__ constexpr int max_threads(int K, int = -1) { return K == 1 ? 1024 : K <= 3 ? 768 : K <= 6 ? 512 : 256; }
 __host__ __device__ constexpr int min_blocks(int) { return 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
 
@@ -699,89 +693,11 @@ __device__ __forceinline__ bool run_blocks(const TB &tb, const uint8_t *p, uint6
 // chains of every active lane coincide the remainder runs ONE chain and its count increments
 // are added to every slot -- bit-identical to running all k chains.  Absent slots start as a copy
 // of slot 0 so they never block the vote (their results are ignored).
-// Two halves (k = 1, latency-bound table variants): a single lookup chain per thread leaves the
-// dependent-load latency exposed (CL: the chain's LDS; G / HS: L2).  The chunk is run as two
-// interleaved halves -- the second half from its own depth-1 look-back guess (A5 top-1) --
-// which doubles the independent chains per thread.  The halves join exactly: if the first half ends
-// in the guess, the second half's run continues it; otherwise the second half is re-executed from
-// the first half's end in lockstep with its guessed chain until the two meet (R3), or to its end.
-template <class TB> struct TableTwoHalves { static constexpr bool value = false; };
-template <> struct TableTwoHalves<TableCL> { static constexpr bool value = true; };
-template <> struct TableTwoHalves<TableB> { static constexpr bool value = true; };
-template <> struct TableTwoHalves<TableG> { static constexpr bool value = true; };
-template <> struct TableTwoHalves<TableHS> { static constexpr bool value = true; };
-constexpr uint64_t kTwoHalvesMin = 256;  // chunk bytes below which the halves do not pay
-
-template <class TB>
-__device__ __forceinline__ void local_phase_halves(const TB &tb, const uint8_t *__restrict__ in, uint64_t b, uint64_t e,
-                                                   uint32_t (&cur)[1], uint32_t (&acc)[1], uint32_t (&accf)[1],
-                                                   uint32_t *stash, const uint16_t *__restrict__ lb)
-{
-    const uint64_t n = e - b;
-    const uint64_t half = (n >> 6) << 5;  // whole sectors, at most half the chunk
-    const uint64_t m = b + half;
-    const uint32_t sB = __ldg(lb + (uint32_t)__ldg(in + m - 1) * KMAX);
-    uint32_t cB[1] = {tb.init(sB)}, aB[1] = {0u}, fB[1] = {0u};
-    const uint8_t *pa = in + b, *pb = in + m;
-    const uint64_t na = half >> 5, nb = (e - m) >> 5;  // na <= nb
-    Bytes32 xa = ldg256(pa), xb = ldg256(pb);
-    if (stash) {
-        reinterpret_cast<uint4 *>(stash)[0] = make_uint4(xa.w[0], xa.w[1], xa.w[2], xa.w[3]);
-        reinterpret_cast<uint4 *>(stash)[1] = make_uint4(xa.w[4], xa.w[5], xa.w[6], xa.w[7]);
-    }
-#pragma unroll 1
-    for (uint64_t i = 0; i < nb; i++) {
-        Bytes32 ya, yb;
-        if (i + 1 < na) ya = ldg256(pa + 32 * (i + 1));
-        if (i + 1 < nb) yb = ldg256(pb + 32 * (i + 1));
-        if (i < na) process32<1>(tb, xa, cur, acc, accf);
-        process32<1>(tb, xb, cB, aB, fB);
-        xa = ya;
-        xb = yb;
-    }
-    for (uint64_t t = m + (nb << 5); t < e; t++) tb.template step<1>(__ldg(in + t), 0, cB, aB, fB);
-    const uint32_t aEnd = tb.state_of(cur[0]);
-    const uint32_t cA = tb.count_of(acc[0], accf[0], cur[0], half), cBn = tb.count_of(aB[0], fB[0], cB[0], e - m);
-    if (aEnd == sB) {
-        cur[0] = cB[0];
-        acc[0] = cA + cBn;
-        accf[0] = 0;
-        return;
-    }
-    uint32_t x = aEnd, y = sB, cx = 0, cy = 0;
-    uint64_t pos = m;
-    const uint64_t wend = min(e, m + kLockstepWindow);
-    bool met = false;
-    while (pos < wend && !met) {
-        const typename TB::Row r = tb.row(__ldg(in + pos));
-        x = tb.apply(r, x, cx);
-        y = tb.apply(r, y, cy);
-        pos++;
-        met = x == y;
-    }
-    if (met) {
-        cur[0] = cB[0];
-        acc[0] = cA + cx - cy + cBn;
-    } else {
-        for (; pos < e; pos++) x = tb.apply(tb.row(__ldg(in + pos)), x, cx);
-        cur[0] = tb.init(x);
-        acc[0] = cA + cx;
-    }
-    accf[0] = 0;
-}
-
 template <int K, class TB>
 __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restrict__ in, uint64_t b, uint64_t e,
                                             bool aligned, uint32_t (&cur)[K], uint32_t (&acc)[K],
-                                            uint32_t (&accf)[K], uint32_t *stash = nullptr,
-                                            const uint16_t *lb = nullptr)
+                                            uint32_t (&accf)[K], uint32_t *stash = nullptr)
 {
-    if constexpr (K == 1 && TableTwoHalves<TB>::value) {
-        if (lb && aligned && !(b & 31) && e - b >= kTwoHalvesMin) {
-            local_phase_halves(tb, in, b, e, cur, acc, accf, stash, lb);
-            return;
-        }
-    }
     if (aligned && (b & 31)) {
         // the peeled head of an unaligned input (chunk 0 starts at in + head): bytes up to the first
         // 32-byte boundary one at a time, then full sectors
@@ -1694,7 +1610,7 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
             accf[s] = 0;
         }
         uint32_t *const stash_j = SPLIT ? nullptr : reinterpret_cast<uint32_t *>(smem + L.stash) + j * 8;
-        if (!empty && e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf, stash_j, p.lb);
+        if (!empty && e > b) local_phase<K>(tb, p.in, b, e, p.aligned != 0, cur, acc, accf, stash_j);
         uint32_t eob[K], cnt[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {

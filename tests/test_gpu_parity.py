@@ -547,7 +547,7 @@ def test_full_geometry_parity(var, n, m):
     """Every table variant at the bench's launch geometry (inputs large enough that pick_geometry
     chooses the maximal tile and 4 KiB chunks, split kernels where the policy splits) against the
     oracle, k = 1 and 2, with the default look-back and eager completion."""
-    L = 640 << 20
+    L = 1280 << 20  # >= 148 SMs x 2 x 1024 threads x 4 KiB: the maximal tile and 4 KiB chunks
     if var == "CL":
         d = dfas.html_tokenizer()
         data = streams.html_bytes(L, 21)

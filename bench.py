@@ -224,6 +224,7 @@ def cpu_model():
 
 def config_json(args, w):
     return {"workload": w["name"], "input_bytes": w["total"], "k": w["k"], "lookback_len": w.get("lookback"),
+            "input_offset": args.offset,
             "eager_window": w.get("eager", 0),
             "n_states": int(w["dfa"].n_states), "parallelism": f"shard{args.gpus}",
             "l2": "input >> L2 (126 MB), no flush needed" if w["total"] > 4 * 126e6 else "L2 flushed between steps"}
@@ -281,6 +282,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-certify", action="store_true", help="skip the full-length certificate (C5)")
     ap.add_argument("--variant", type=int, default=-1)
+    ap.add_argument("--offset", type=int, default=0,
+                    help="start the input this many bytes past a 32-byte boundary (unaligned-input path, R10)")
     ap.add_argument("--lookback", type=int, default=-1,
                     help="look-back window bytes (R7; -1 = the config's default: c5 0, c1/c4 64, c2/c3 32)")
     ap.add_argument("--chunk", type=int, default=0)
@@ -327,7 +330,9 @@ def main():
     hi = total if rank == world - 1 else total * (rank + 1) // world // 32 * 32
     n = hi - lo
     nsym = n * 8 if w["bits"] else n   # the library counts symbols: bits in bit mode
-    buf = torch.empty(n + 64, dtype=torch.uint8, device=dev)
+    off = args.offset
+    base = torch.empty(n + 64 + off, dtype=torch.uint8, device=dev)
+    buf = base[off:]  # buf.data_ptr() is base + off: unaligned when off % 32 != 0
     halo = torch.zeros(32, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
     if "data" in w:
@@ -507,7 +512,7 @@ def main():
                 flush.zero_()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            rc = _native.dev_lib().fsmgen_dev_read_stream(buf.data_ptr(), n, sink.data_ptr(),
+            rc = _native.dev_lib().fsmgen_dev_read_stream(base.data_ptr(), n, sink.data_ptr(),
                                                           torch.cuda.get_device_properties(dev).multi_processor_count,
                                                           stream.cuda_stream)
             e1.record(stream)

@@ -341,6 +341,13 @@ typedef struct {
 
 int fsm_debug_get_merge(const fsm_t *f, fsm_debug_merge *out);
 
+/* fsm_hot_state_order: the static frequency order of hot-state caching (Sec. 4.2; NEXT-1),
+ * host only: user state ids sorted by in-degree in the byte-level transition table (bit mode: the
+ * widened table) descending, ties to the smaller id.  The HS variant keeps the rows of a prefix of
+ * this order in shared memory.  order_out: n_states entries.  Errors: FSM_EINVAL. */
+int fsm_hot_state_order(const uint32_t *table, uint32_t n_states, uint32_t alphabet, uint32_t input_mode,
+                        uint32_t *order_out);
+
 /* Library version string. */
 const char *fsm_version(void);
 

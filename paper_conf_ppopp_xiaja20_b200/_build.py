@@ -27,28 +27,47 @@ def stale() -> bool:
     return any(os.path.getmtime(s) > t for s in sources())
 
 
+OBJ = os.path.join(HERE, "build")  # per-unit objects (git-ignored), reused when their inputs are unchanged
+
+
+def _unit_stale(u: str, obj: str) -> bool:
+    """A kernel unit depends on its .cu and every header; fsmspec.cu (host side) on itself, the
+    headers and the public header.  Host-only edits therefore relink without recompiling kernels."""
+    if not os.path.exists(obj):
+        return True
+    deps = [os.path.join(CSRC, u + ".cu")] + glob.glob(os.path.join(CSRC, "*.cuh")) + \
+        glob.glob(os.path.join(CSRC, "*.h")) + [os.path.join(ROOT, "include", "fsmspec.h"), __file__]
+    t = os.path.getmtime(obj)
+    return any(os.path.getmtime(d) > t for d in deps)
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     """Compile the translation units in parallel (one per table variant) and link the .so."""
     if not force and not stale():
         return SO
     import concurrent.futures as cf
-    import tempfile
 
-    tmp = tempfile.mkdtemp(prefix="fsmspec_build_")
+    os.makedirs(OBJ, exist_ok=True)
     log = os.path.join(HERE, "build.log")
+    extra = os.environ.get("FSMSPEC_EXTRA_FLAGS", "").split()  # experiments only
 
     def unit(u):
-        obj = os.path.join(tmp, u + ".o")
-        extra = os.environ.get("FSMSPEC_EXTRA_FLAGS", "").split()  # experiments only
+        obj = os.path.join(OBJ, u + ".o")
         cmd = [NVCC, *FLAGS, *extra, "-I", os.path.join(ROOT, "include"), "-c", "-o", obj, os.path.join(CSRC, u + ".cu")]
+        if not (force or extra) and not _unit_stale(u, obj):
+            return u, obj, cmd, None
         res = subprocess.run(cmd, capture_output=True, text=True)
+        if res.returncode != 0 and os.path.exists(obj):
+            os.remove(obj)
         return u, obj, cmd, res
 
     with cf.ThreadPoolExecutor(len(UNITS)) as ex:
         results = list(ex.map(unit, UNITS))
-    with open(log, "w") as fh:
+    with open(log, "a" if not force else "w") as fh:
         for u, obj, cmd, res in results:
-            fh.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
+            if res is not None:
+                fh.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
+    results = [(u, o, c, r if r is not None else subprocess.CompletedProcess(c, 0, "", "")) for u, o, c, r in results]
     bad = [(u, r) for u, _, _, r in results if r.returncode != 0]
     if bad:
         raise RuntimeError(f"nvcc failed for {bad[0][0]} (see {log}):\n{bad[0][1].stderr[-4000:]}")
@@ -58,9 +77,6 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if res.returncode != 0:
         raise RuntimeError(f"link failed:\n{res.stderr[-4000:]}")
     os.replace(SO + ".tmp", SO)
-    import shutil
-
-    shutil.rmtree(tmp, ignore_errors=True)
     if verbose:
         print(open(log).read()[-2000:])
     return SO

@@ -238,6 +238,21 @@ extern "C" int fsm_lookback_table(const uint32_t *table, uint32_t n_states, uint
     return FSM_OK;
 }
 
+extern "C" int fsm_hot_state_order(const uint32_t *table, uint32_t n_states, uint32_t alphabet, uint32_t input_mode,
+                                   uint32_t *order_out)
+{
+    if (!table || !order_out || n_states == 0 || alphabet == 0 || alphabet > 256) return FSM_EINVAL;
+    if (input_mode == FSM_INPUT_BITS_MSB && alphabet != 2) return FSM_EINVAL;
+    for (size_t i = 0; i < (size_t)n_states * alphabet; i++)
+        if (table[i] >= n_states) return FSM_EINVAL;
+    ByteDFA d;
+    build_byte_dfa(table, n_states, alphabet, nullptr, input_mode == FSM_INPUT_BITS_MSB, d);
+    std::vector<uint32_t> perm, inv;
+    renumber_by_frequency(d, n_states, perm, inv);
+    for (uint32_t r = 0; r < n_states; r++) order_out[r] = inv[r];
+    return FSM_OK;
+}
+
 static void free_all(fsm *f)
 {
     for (int i = 0; i < 9; i++) cudaFree(f->d_img[i]);

@@ -30,7 +30,7 @@ EXPORTS = ("fsm_create", "fsm_create_ex", "fsm_destroy", "fsm_strerror", "fsm_se
            "fsm_run_spec_k", "fsm_run_spec_k_async", "fsm_run_spec_k_host", "fsm_set_options",
            "fsm_get_options", "fsm_get_stats", "fsm_run_shard", "fsm_shard_fixup", "fsm_shard_free",
            "fsm_map_compose", "fsm_compose_from", "fsm_lookback_table", "fsm_version", "fsm_autotune",
-           "fsm_run_multi", "fsm_debug_set_spec", "fsm_debug_get_merge")
+           "fsm_run_multi", "fsm_debug_set_spec", "fsm_debug_get_merge", "fsm_hot_state_order")
 
 
 class fsm_options(ctypes.Structure):
@@ -128,6 +128,7 @@ def lib() -> ctypes.CDLL:
                                        ctypes.POINTER(fsm_shard_map)]),
             "fsm_lookback_table": (_I32, [_P, _U32, _U32, _U32, _P, _P]),
             "fsm_version": (ctypes.c_char_p, []),
+            "fsm_hot_state_order": (_I32, [_P, _U32, _U32, _U32, _P]),
             "fsm_compose_from": (_I32, [ctypes.POINTER(fsm_shard_map), _U32, _U32, _U64, ctypes.POINTER(_U32),
                                         ctypes.POINTER(_U64), ctypes.POINTER(_U32)]),
             "fsm_debug_set_spec": (_I32, [_P, _P, _U32, _U32, _U32]),
@@ -171,6 +172,16 @@ def lookback_table(table: np.ndarray, bit_mode: bool = False):
                                     FSM_INPUT_BITS_MSB if bit_mode else FSM_INPUT_BYTES,
                                     lb.ctypes.data, ni.ctypes.data), "fsm_lookback_table")
     return lb, ni
+
+
+def hot_state_order(table: np.ndarray, bit_mode: bool = False) -> list[int]:
+    """fsm_hot_state_order (host only): states by static in-degree, the hot-state caching order."""
+    t = np.ascontiguousarray(table, dtype=np.uint32)
+    out = np.zeros(t.shape[0], np.uint32)
+    _check(lib().fsm_hot_state_order(t.ctypes.data, t.shape[0], t.shape[1],
+                                     FSM_INPUT_BITS_MSB if bit_mode else FSM_INPUT_BYTES, out.ctypes.data),
+           "fsm_hot_state_order")
+    return [int(x) for x in out]
 
 
 def map_compose(a: fsm_shard_map, b: fsm_shard_map) -> fsm_shard_map:

@@ -140,3 +140,25 @@ def test_variant_enum_matches_header():
     assert {v: k for k, v in enum.items()} == fsmspec.VARIANT_NAMES
     for name, v in enum.items():
         assert getattr(fsmspec, "FSM_VARIANT_" + name) == v
+
+
+def test_hot_state_order_p5(golden):
+    """P5: the static frequency of Fig. 1b is a = c = 4, b = d = 2, so with 6 shared-
+    memory entries (two rows of three symbols) the rows of a and c are cached.  The library's own
+    hot-state caching order (the HS variant's renumbering) must put a and c first, for the
+    3-symbol table and for the 256-column expansion alike."""
+    g = golden["c_comment_fig1"]
+    names = g["states"]
+    for expanded in (False, True):
+        d = dfas.c_comment(expanded=expanded)
+        order = fsmspec.hot_state_order(d.table)
+        rows = 6 // 3                                                       # P:235: 6 entries
+        assert {names[s] for s in order[:rows]} == set(g["hot_rows_6_entries"]["rows"]), expanded
+        assert sorted(order) == list(range(4))
+    # in-degree ranking against an independent count on random tables (ties -> smaller id)
+    rng = np.random.default_rng(5)
+    for _ in range(5):
+        t = rng.integers(0, 12, (12, 256)).astype(np.uint32)
+        indeg = np.bincount(t.ravel(), minlength=12)
+        exp = sorted(range(12), key=lambda s: (-indeg[s], s))
+        assert fsmspec.hot_state_order(t) == exp

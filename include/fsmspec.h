@@ -149,9 +149,11 @@ typedef struct {
                                    candidates (rank order) are re-executed before publishing, so a
                                    successor passes through them without waiting; the others are
                                    published invalid and re-executed only if the true path enters the
-                                   tile in them.  0 = default (FSM_PRERESOLVE_DEFAULT), 1..FSM_KMAX =
-                                   top n (n >= k: every slot), FSM_PRERESOLVE_NONE = only the true path
-                                   is ever re-executed.  Results are identical under every setting. */
+                                   tile in them.  0 = default: the top candidate only, or every
+                                   candidate when every symbol permutes the states (paths never meet,
+                                   so a lazily resolved candidate is a whole-chunk re-execution chain);
+                                   1..FSM_KMAX = top n (n >= k: every slot); FSM_PRERESOLVE_NONE = only
+                                   the true path is ever re-executed.  Identical results. */
     uint32_t grid_sms;          /* SMs the persistent grids use (0 = all): the grid-size sweep of the
                                    sequential- vs parallel-merge ablation (Figs. 7-11 vary the number of
                                    thread blocks) */
@@ -254,7 +256,8 @@ int fsm_compose_from(const fsm_shard_map *maps, uint32_t n, uint32_t start_state
  * default window (64 bytes, eager on) and with the paper's depth-1 look-back (eager off); (2) for
  * the two fastest k, look-back windows {0, 32, 64, 128, 256} x eager {off, 128}; (3) for the chosen
  * setting, every table variant the DFA fits (the by-size default is a heuristic: e.g. a random
- * 1024-state DFA runs faster with hot-state caching, a 1027-state Aho-Corasick DFA without).
+ * 1024-state DFA runs faster with hot-state caching, a 1027-state Aho-Corasick DFA without); (4) for
+ * k > 1, pre-resolution of the top tile-start candidate vs every candidate (fsm_options.preresolve).
  *   input, len   device pointer and length (symbols) of the input the runs will process
  *   k_min, k_max smallest / largest k to consider (0 = 1 / min(FSM_KMAX, n_states); k_min = k_max
  *                tunes only the windows for that k)
@@ -274,6 +277,7 @@ typedef struct {
     double paper_gbs;           /* same for the paper's plain setting: k = 1, depth-1 look-back, no eager */
     double hit_rate;            /* 1 - re-executed chunks / chunks, chosen configuration */
     int32_t variant;            /* chosen table variant (FSM_VARIANT_*), applied to the options */
+    uint32_t preresolve;        /* chosen fsm_options.preresolve (0 = the default policy), applied */
 } fsm_tuning;
 
 int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k_min, uint32_t k_max,

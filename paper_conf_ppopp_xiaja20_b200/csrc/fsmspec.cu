@@ -135,6 +135,7 @@ struct fsm {
     uint32_t n_user = 0, alphabet = 0, start = 0, mode = 0;
     ByteDFA dfa;
     int auto_variant = VAR_G;
+    bool permutation = false;  // every in-alphabet symbol permutes the states: paths never meet
     fsm_options opt{};
     // device tables
     void *d_img[9] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
@@ -326,6 +327,20 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         renumber_by_frequency(f->dfa, n_states, f->perm, f->inv);
         f->renumbered = true;
         f->start_int = f->perm[start];
+    }
+    {   // paths of a DFA whose every symbol is a bijection never converge (R5 default below)
+        bool perm = true;
+        const uint32_t ncols = bits ? 256u : alphabet;
+        std::vector<uint8_t> seen(f->dfa.n);
+        for (uint32_t c = 0; c < ncols && perm; c++) {
+            std::fill(seen.begin(), seen.end(), 0);
+            for (uint32_t s = 0; s < n_states && perm; s++) {
+                const uint32_t t = f->dfa.next[(size_t)s * 256 + c];
+                if (t >= n_states || seen[t]) perm = false;
+                else seen[t] = 1;
+            }
+        }
+        f->permutation = perm;
     }
     f->lb.resize(256 * KMAX);
     f->nimg.resize(256);
@@ -524,12 +539,15 @@ constexpr int kMultiMaxK = 8;  // fused multi-FSM kernels are instantiated for K
 // tile size, else Alg. 1 (measured on B200: the hash form wins where the tile keeps
 // its size, e.g. 64-state B k = 16 +12 %, and loses where the tile must halve, e.g. HTML CL -26 %)
 constexpr bool kHashAuto = true;
-// R5 default (fsm_options.preresolve = 0): see DESIGN.md "R5".
-constexpr uint32_t kPreresolveDefault = 1;
+// R5 default (fsm_options.preresolve = 0), measured: the top-ranked tile-start
+// candidate only -- except for DFAs whose paths never meet (every symbol a permutation), where a
+// lazily resolved candidate costs a whole-chunk re-execution chain on the look-back's critical
+// path, so every candidate is pre-resolved in parallel.
 static uint32_t preresolve_of(const fsm *f)
 {
     const uint32_t v = f->opt.preresolve;
-    return v == 0 ? kPreresolveDefault : v == FSM_PRERESOLVE_NONE ? 0u : v;
+    if (v == 0) return f->permutation ? (uint32_t)FSM_KMAX : 1u;
+    return v == FSM_PRERESOLVE_NONE ? 0u : v;
 }
 
 // Chunks per tile: a split kernel (split_kernel(var, K)) gives the CTA's last warp to the epilogue.
@@ -1195,6 +1213,7 @@ namespace {
 struct TuneCand {
     uint32_t k, lookback, eager;
     int32_t variant = FSM_VARIANT_AUTO;
+    uint32_t preresolve = 0;
     double ms = 0, hit = 0;
 };
 }  // namespace
@@ -1206,6 +1225,7 @@ static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom
     o.lookback_len = c.lookback;
     o.eager_window = c.eager;
     o.variant = c.variant;
+    o.preresolve = c.preresolve;
     o.merge = FSM_MERGE_PARALLEL;
     int rc = fsm_set_options(f, &o);
     if (rc) return rc;
@@ -1249,11 +1269,11 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
     CK(cudaEventCreate(&e1));
     std::vector<TuneCand> tried;
     int rc = FSM_OK;
-    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg, int32_t var = -2) -> int {
+    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg, int32_t var = -2, uint32_t pre = 0) -> int {
         if (var == -2) var = saved.variant;  // stages 1-2: the handle's own variant choice
         for (const TuneCand &c : tried)
-            if (c.k == k && c.lookback == lb && c.eager == eg && c.variant == var) return FSM_OK;
-        TuneCand c{k, lb, eg, var};
+            if (c.k == k && c.lookback == lb && c.eager == eg && c.variant == var && c.preresolve == pre) return FSM_OK;
+        TuneCand c{k, lb, eg, var, pre};
         int r = time_candidate(f, input, n, len / sym_per_byte, c, e0, e1);
         if (r == FSM_OK) tried.push_back(c);
         return r;
@@ -1292,6 +1312,16 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
         for (int v = 0; v < 9 && rc == FSM_OK; v++)
             if (f->d_img[v] && v != base) rc = run(best_so_far.k, best_so_far.lookback, best_so_far.eager, v);
     }
+    // stage 4: R5 pre-resolution (top-1 vs every candidate) at the best setting so far
+    if (rc == FSM_OK) {
+        const TuneCand *b = nullptr;
+        for (const TuneCand &c : tried)
+            if (c.k >= k_min && c.k <= k_max && (!b || c.ms < b->ms)) b = &c;
+        const TuneCand bb = *b;
+        if (bb.k > 1)
+            for (uint32_t pre : {1u, (uint32_t)FSM_KMAX})
+                if (rc == FSM_OK) rc = run(bb.k, bb.lookback, bb.eager, bb.variant, pre);
+    }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     f->opt = saved;
@@ -1313,9 +1343,11 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
     out->hit_rate = best->hit;
     out->variant = best->variant != FSM_VARIANT_AUTO ? best->variant
                  : saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;
+    out->preresolve = best->preresolve;
     f->opt.lookback_len = best->lookback;
     f->opt.eager_window = out->eager_window;
     f->opt.variant = out->variant;
+    f->opt.preresolve = best->preresolve;
     return FSM_OK;
 }
 

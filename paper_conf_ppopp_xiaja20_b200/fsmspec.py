@@ -43,7 +43,8 @@ class fsm_options(ctypes.Structure):
 class fsm_tuning(ctypes.Structure):
     _fields_ = [("k", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32),
                 ("candidates", ctypes.c_uint32), ("sample_len", ctypes.c_uint64), ("best_gbs", ctypes.c_double),
-                ("paper_gbs", ctypes.c_double), ("hit_rate", ctypes.c_double), ("variant", ctypes.c_int32)]
+                ("paper_gbs", ctypes.c_double), ("hit_rate", ctypes.c_double), ("variant", ctypes.c_int32),
+                ("preresolve", ctypes.c_uint32)]
 
 
 class fsm_stats(ctypes.Structure):

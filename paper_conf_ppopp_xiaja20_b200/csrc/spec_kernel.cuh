@@ -47,13 +47,6 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
                     cur[q0][i] = tb.init((uint32_t)__ldg(p.lb + c0 * KMAX + ((uint32_t)ii < ni ? ii : 0)));
                     acc[q0][i] = accf[q0][i] = 0;
                 }
-            // Paths that meet stay together: every 16 bytes a group whose four chains all equal chains
-            // of earlier live groups is frozen (its chains follow their twins from then on), so the
-            // window costs about one group per chunk once the image has converged.
-            uint32_t live = 0, twin[KMAX / 4] = {0u, 0u, 0u, 0u};
-#pragma unroll
-            for (int q0 = 0; q0 < KMAX / 4; q0++)
-                if ((uint32_t)(q0 * 4) < ni) live |= 1u << q0;
             for (uint32_t o = 0; o < Lw; o += 32) {
                 const Bytes32 x = ldg256(p.in + b - Lw + o);
 #pragma unroll
@@ -62,35 +55,7 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
                     for (int j = 0; j < 4; j++)
 #pragma unroll
                         for (int q0 = 0; q0 < KMAX / 4; q0++)
-                            if ((live >> q0) & 1u) tb.template step<4>(x.w[q], j, cur[q0], acc[q0], accf[q0]);
-                    if ((q & 3) == 3 && live > 1u) {
-                        uint32_t sv[KMAX];
-#pragma unroll
-                        for (int q0 = 0; q0 < KMAX / 4; q0++)
-#pragma unroll
-                            for (int i = 0; i < 4; i++) sv[q0 * 4 + i] = tb.state_of(cur[q0][i]);
-#pragma unroll
-                        for (int g = 1; g < KMAX / 4; g++) {
-                            if (!((live >> g) & 1u)) continue;
-                            uint32_t tw = 0;
-                            bool all = true;
-#pragma unroll
-                            for (int i = 0; i < 4; i++) {
-                                int f = -1;
-#pragma unroll
-                                for (int h = 0; h < g; h++)
-#pragma unroll
-                                    for (int l = 0; l < 4; l++)
-                                        if (f < 0 && ((live >> h) & 1u) && sv[h * 4 + l] == sv[g * 4 + i]) f = h * 4 + l;
-                                all = all && f >= 0;
-                                tw |= (uint32_t)(f & 15) << (4 * i);
-                            }
-                            if (all) {
-                                live &= ~(1u << g);
-                                twin[g] = tw;
-                            }
-                        }
-                    }
+                            if ((uint32_t)(q0 * 4) < ni) tb.template step<4>(x.w[q], j, cur[q0], acc[q0], accf[q0]);
                 }
             }
             uint32_t y[KMAX];
@@ -98,19 +63,6 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
             for (int q0 = 0; q0 < KMAX / 4; q0++)
 #pragma unroll
                 for (int i = 0; i < 4; i++) y[q0 * 4 + i] = tb.state_of(cur[q0][i]);
-#pragma unroll
-            for (int g = 1; g < KMAX / 4; g++)  // frozen groups take their twins' end states (in order)
-                if ((uint32_t)(g * 4) < ni && !((live >> g) & 1u)) {
-#pragma unroll
-                    for (int i = 0; i < 4; i++) {
-                        const uint32_t t = (twin[g] >> (4 * i)) & 15u;
-                        uint32_t v = 0;
-#pragma unroll
-                        for (int l = 0; l < KMAX; l++)
-                            if ((uint32_t)l == t) v = y[l];
-                        y[g * 4 + i] = v;
-                    }
-                }
             uint32_t mult[KMAX];
 #pragma unroll
             for (int i = 0; i < KMAX; i++) {

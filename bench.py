@@ -275,7 +275,8 @@ def main():
     ap.add_argument("--k-override", type=int, default=0, help="k for c1-c4 (c5 uses --k)")
     ap.add_argument("--ac-states", type=int, default=1024, help="c3: minimum Aho-Corasick states (1024 / 4096)")
     ap.add_argument("--n-states", type=int, default=8)
-    ap.add_argument("--m", type=int, default=2)
+    ap.add_argument("--image", "--m", dest="m", type=int, default=2,
+                    help="C5: |image(c)| of the random DFA (--image under torchrun: --m is ambiguous there)")
     ap.add_argument("--k", type=int, default=2)
     ap.add_argument("--size-gib", type=float, default=0.0, help="input size (default: the config's)")
     ap.add_argument("--no-e2e", action="store_true")

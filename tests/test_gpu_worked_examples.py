@@ -254,3 +254,43 @@ def test_hash_check_merge_tree_identical():
             out[chk] = [[m.mapping(lv, lane) for lane in range(32)] for lv in range(6)]
             out[chk].append([[int(m.brk[lv][lane][s]) for s in range(16)] for lv in range(6) for lane in range(32)])
     assert out[fsmspec.FSM_CHECK_NESTED] == out[fsmspec.FSM_CHECK_HASH]
+
+
+# --------------------------------------------------------------------- randomised merge trees vs the CPU model
+@pytest.mark.parametrize("seed", range(4))
+def test_random_injected_merge_trees(seed):
+    """Tiny random DFAs (N <= 4, 2 symbols), random inputs of up to 32 chunks of 1-4 bytes and random
+    injected speculated sets (chunk 0's may miss q0): every warp-scan level read back from the GPU
+    equals the CPU model's merge (oracle/speck.py, Sec. 3.3) of the same chunks, slot by
+    slot and validity included, and the result equals the oracle.  ~400 cases per seed."""
+    rng = np.random.default_rng(1000 + seed)
+    cases = 0
+    while cases < 400:
+        n = int(rng.integers(2, 5))
+        table = rng.integers(0, n, (n, 2)).astype(np.uint32)
+        acc = rng.integers(0, 2, n).astype(np.uint8)
+        d = dfas.DFA(table, int(rng.integers(0, n)), acc, False, "tiny")
+        c = int(rng.integers(1, 5))
+        nch = int(rng.integers(1, 33))
+        L = c * (nch - 1) + int(rng.integers(1, c + 1))
+        data = rng.integers(0, 2, L).astype(np.uint8)
+        k = int(rng.integers(1, n + 1))
+        sets = [list(rng.choice(n, int(rng.integers(1, k + 1)), replace=False)) for _ in range(nch)]
+        with FSM.from_dfa(d) as f:
+            f.set_options(eager_window=fsmspec.FSM_EAGER_OFF)
+            f.debug_set_spec([[int(x) for x in s_] for s_ in sets], chunk_bytes=c, k=k)
+            buf, ptr = dev(data)
+            got = f.run_spec_k(ptr, L, k)
+            m = f.debug_get_merge()
+        assert got == seq.run(d, data), (seed, cases)
+        bounds = [min(j * c, L) for j in range(nch)] + [L]
+        maps = speck.local_phase(d, [int(x) for x in data], bounds, sets)
+        level = list(maps)
+        for lv in range(6):
+            for j in range(nch):
+                exp = {s: (None if e is None else (e, cnt)) for s, e, cnt in zip(level[j].starts, level[j].ends,
+                                                                                   level[j].counts)}
+                assert m.mapping(lv, j) == exp, (seed, cases, lv, j)
+            step = 1 << lv
+            level = [speck.merge(level[j], level[j + step]) if j + step < nch else level[j] for j in range(nch)]
+        cases += 1

@@ -714,10 +714,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     p.k_1e24 = 1u << 24;
     p.k_16 = 16;
     p.k_512 = 512;
-    p.k_1e27 = 1u << 27;
-    p.k_2 = 2;
     p.k_4 = 4;
-    p.k_1e28 = 1u << 28;
     p.table_g = static_cast<const uint32_t *>(f->d_img[VAR_G]);
     p.hot_rows = f->hot_rows;
     p.inv = f->d_inv;
@@ -1062,8 +1059,8 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         fp.bittab = f->d_bittab;
         fp.out = f->d_fix;
         fp.stats = f->d_stats;
-        fp.kc = KConst{1u << 24, 16, 512, 1u << 27, 2, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows,
-                       f->ncls, f->cl_magic, 4, 1u << 28};
+        fp.kc = KConst{1u << 24, 16, 512, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows, f->ncls,
+                       f->cl_magic, 4};
         FixFn fn = get_fix(var);
         const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
         CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

@@ -159,15 +159,15 @@ __device__ __forceinline__ void check_smem_window(int var, uint32_t need)
 }
 
 struct KConst {
-    uint32_t k_1e24, k_16, k_512, k_1e27, k_2;
+    uint32_t k_1e24, k_16, k_512;
     const uint32_t *gtab;  // full u32 table in global memory (HS variant)
     uint32_t hot_rows;     // HS: states [0, hot_rows) have their rows in shared memory
     uint32_t ncls, cl_magic;  // CL: byte classes, ceil(2^32 / ncls)
-    uint32_t k_4, k_1e28;     // N8
+    uint32_t k_4;             // N8
 };
 __device__ __forceinline__ KConst kconst(const Params &p)
 {
-    return KConst{p.k_1e24, p.k_16, p.k_512, p.k_1e27, p.k_2, p.table_g, p.hot_rows, p.ncls, p.cl_magic, p.k_4, p.k_1e28};
+    return KConst{p.k_1e24, p.k_16, p.k_512, p.table_g, p.hot_rows, p.ncls, p.cl_magic, p.k_4};
 }
 
 // ------------------------------------------------------------------- table-placement variants --
@@ -1023,17 +1023,11 @@ __device__ __forceinline__ void named_arrive(uint32_t id, uint32_t n)
 // (HTML, k = 1: +13 %, its serial re-executions dominate the epilogue) and the multi-chain kernels
 // of the shared-memory variants (P4 / P8 / B, K >= 2: +6..15 %).  K = 1 kernels of P8 / B / G / HS
 // lose more from the missing 32nd worker warp and stash than they gain (-4..-8 %): unsplit.
-// FSM_SPLIT: 2 = this policy (default), 1 = always, 0 = never (experiments).  A launch runs split
-// only if the policy says so AND the double-buffered layout fits in shared memory (large-K CL
-// kernels next to a 150 KiB table do not).
-#ifndef FSM_SPLIT
-#define FSM_SPLIT 2
-#endif
+// A launch runs split only if this policy says so AND the double-buffered layout fits in shared
+// memory (large-K CL kernels next to a 150 KiB table do not).
 __host__ __device__ constexpr bool split_kernel(int var, int K)
 {
-    return FSM_SPLIT == 1 ? true
-         : FSM_SPLIT == 0 ? false
-         : (var == 6 /* CL */ || ((var == 0 || var == 1 || var == 2 || var == 7 || var == 8) /* P4 P8 B N8 R16 */ && K >= 2));
+    return var == 6 /* CL */ || ((var == 0 || var == 1 || var == 2 || var == 7 || var == 8) /* P4 P8 B N8 R16 */ && K >= 2);
 }
 
 // Per-tile context used by re-execution and the epilogue.
@@ -1049,7 +1043,6 @@ struct TileCtx {
     const uint16_t *Sj;
     const uint32_t *stash;  // first 32 bytes of every chunk (valid when aligned and >= 32 bytes)
     const uint32_t *ext;    // eager-completion entries, kExt per chunk
-    DevStats *stats;
 };
 
 // Look up an eager-completion entry of chunk c for state st: returns the slot (or -1) and delta.
@@ -1247,7 +1240,6 @@ __device__ __forceinline__ void tile_epilogue(const TB &tb, const Params &p, uin
     t.Sj = Sj;
     t.stash = stash;
     t.ext = Ext;
-    t.stats = p.stats;
 
     // a8 (tile candidates, R5): resolve the broken slots of the tile aggregate Q_0 for the top
     // p.preresolve speculated tile starts, so that a successor's look-back can pass through them
@@ -1599,9 +1591,6 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
         speculate<K>(tb, p, b, first_chunk, empty, start_state, S, Xc);
 
         // ---- a4: local processing
-#ifdef FSM_PHASE_TIMING
-        long long t_local0 = clock64();
-#endif
         uint32_t cur[K], acc[K], accf[K];
 #pragma unroll
         for (int s = 0; s < K; s++) {
@@ -1678,10 +1667,6 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
         }
         bool ident = empty;
 
-#ifdef FSM_PHASE_TIMING
-        long long t_local1 = clock64();
-        atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 40, (unsigned long long)(t_local1 - t_local0));
-#endif
         // ---- a5: warp stage (chunks warp*32 .. warp*32+31)
         __syncwarp();  // the lanes' eager-completion entries are read by the scan
         warp_suffix_scan<K, HASH>(S, eob, cnt, ident, (uint32_t)warp * 32, 1, Ext,
@@ -1746,10 +1731,6 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
         }
         __syncthreads();
 
-#ifdef FSM_PHASE_TIMING
-        long long t_scan1 = clock64();
-        if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long *>(p.result) + 41, (unsigned long long)(t_scan1 - t_local1));
-#endif
         if (warp != 0) continue;
 
         // ================= warp 0: tile epilogue (pre-resolution, look-back, publication) =====

@@ -101,14 +101,14 @@ struct Params {
     DevStats *stats;
     // constants passed at run time so that ptxas cannot strength-reduce the FMA-pipe IMADs into
     // ALU-pipe shifts (the hot loop balances the two pipes): 1 << 24, 16, 512
-    uint32_t k_1e24, k_16, k_512, k_1e27, k_2;
+    uint32_t k_1e24, k_16, k_512;
     const uint32_t *table_g;       // full u32 table (HS variant's cold rows)
     uint32_t hot_rows;             // HS variant: rows cached in shared memory
     const uint32_t *inv;           // internal -> user state ids (renumbered handles), or null
     uint32_t ncls, cl_magic;       // CL variant: byte classes and ceil(2^32 / ncls)
     uint32_t *user_out;            // optional: the last tile also writes {user state, 0, count lo, hi} here
     uint32_t eager_window;         // NEXT-3 eager completion: bytes of lockstep per chunk (0 = off)
-    uint32_t k_4, k_1e28;          // N8 variant: FMA-pipe constants (4, 1 << 28), see k_1e24 above
+    uint32_t k_4;                  // N8 variant: FMA-pipe constant 4, see k_1e24 above
     uint32_t preresolve;           // R5: tile-start slots (in rank order) resolved before publishing A
     uint32_t spec_all;             // test hook: `spec` also overrides chunk 0 of a known-start run
     uint4 *dbg;                    // test hook: warp-scan levels of tile 0, warp 0 ([6][32][KMAX]), or null

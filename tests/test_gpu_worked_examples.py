@@ -294,3 +294,20 @@ def test_random_injected_merge_trees(seed):
             step = 1 << lv
             level = [speck.merge(level[j], level[j + step]) if j + step < nch else level[j] for j in range(nch)]
         cases += 1
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 5, 7])
+def test_div7_reexecution_rate_is_one_minus_k_over_7(k):
+    """Div7 on random bits: the widened-byte look-back image is all 7 states with equal
+    weight, so a chunk's true start is speculated with probability k/7 and the GPU's true-path
+    re-execution rate must approach 1 - k/7; k = 7 (spec-N) never re-executes."""
+    d = dfas.div7()
+    n_bits = 8 * (32 << 20)
+    data = streams.random_bits(n_bits, seed=70 + k)
+    with FSM.from_dfa(d) as f:
+        f.set_options(eager_window=fsmspec.FSM_EAGER_OFF, chunk_bytes=1024, variant=VARIANTS["P8"])
+        buf, ptr = dev(data)
+        assert f.run_spec_k(ptr, n_bits, k) == seq.run(d, data, n_bits)
+        st = f.stats()
+    rate = st["reexec_true"] / (st["chunks"] - 1)
+    assert abs(rate - (1 - k / 7)) < 0.01, (k, rate, st)

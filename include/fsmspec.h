@@ -56,12 +56,19 @@ enum {
     /* 4 is retired (H8: half rows, one LDS.32 per chain step -- measured slower than P8 and N8) */
     FSM_VARIANT_HS = 5,  /* byte mode, N <= 32768: hot-state row caching (Sec. 4.2): the most frequent
                             states' rows in shared memory (u16), the rest from the u32 table in L2 */
-    FSM_VARIANT_CL = 6,  /* N x byte-classes <= 1024: class-compressed, lane-replicated table, one
-                            conflict-free LDS.32 per chain step (e.g. the HTML tokenizer) */
+    FSM_VARIANT_CL = 6,  /* byte mode, N x ceil(byte-classes / 2) <= 504: class-compressed, lane-replicated u16
+                            table whose entries are the next row's shared address, one PRMT + LDS for the class,
+                            IADD + conflict-free LDS.U16 per chain step (e.g. the HTML tokenizer)       */
     FSM_VARIANT_N8 = 7,  /* N <= 8 (byte mode): one u32 row of eight 4-bit fields per symbol, lane-replicated
                             smem (one LDS.32 per byte), chain = wrap-mode funnel shift + IMAD          */
-    FSM_VARIANT_R16 = 8  /* N <= 16: byte entries (next | count << 4), lane-replicated so that lane l reads
-                            bank l (128 KiB smem at N = 16), one conflict-free LDS.U8 per chain step  */
+    FSM_VARIANT_R16 = 8, /* N <= 16 (byte mode): byte entries (bare next state), lane-replicated so that lane
+                            l reads bank l (128 KiB smem at N = 16), IMAD + conflict-free LDS.U8 per chain
+                            step.  R16 and CL count accepts by region: byte-mode handles renumber their
+                            states internally so that F (or its complement) is the top id range; results,
+                            maps and debug readbacks are always in the caller's ids                   */
+    FSM_VARIANT_RG = 9   /* N <= 256 (byte mode): R16's layout in 32 >> logl copies (lanes 2^logl g ..
+                            share copy g, which owns banks of its own; logl = smallest with the table
+                            <= 128 KiB): a warp's LDS.U8 costs the worst bank load of 2^logl lanes     */
 };
 
 /* Merge strategies: the paper's parallel merge (default) and its sequential-merge baseline

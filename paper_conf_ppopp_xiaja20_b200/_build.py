@@ -12,7 +12,7 @@ SO = os.environ.get("FSMSPEC_BUILD_SO") or os.path.join(HERE, "libfsmspec.so")  
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
-UNITS = ["fsmspec", "kernels_p4", "kernels_p8", "kernels_b", "kernels_g", "kernels_hs", "kernels_cl", "kernels_n8", "kernels_r16"]
+UNITS = ["fsmspec", "kernels_p4", "kernels_p8", "kernels_b", "kernels_g", "kernels_hs", "kernels_cl", "kernels_n8", "kernels_r16", "kernels_rg"]
 
 
 def sources() -> list[str]:

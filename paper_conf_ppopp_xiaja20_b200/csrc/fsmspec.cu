@@ -52,6 +52,7 @@ FSM_DECLARE_VARIANT(hs)
 FSM_DECLARE_VARIANT(cl)
 FSM_DECLARE_VARIANT(n8)
 FSM_DECLARE_VARIANT(r16)
+FSM_DECLARE_VARIANT(rg)
 
 static KernelFn get_kernel(int var, int K, bool split, bool hash)
 {
@@ -62,6 +63,7 @@ static KernelFn get_kernel(int var, int K, bool split, bool hash)
     case VAR_CL: return get_kernel_cl(K, split, hash);
     case VAR_N8: return get_kernel_n8(K, split, hash);
     case VAR_R16: return get_kernel_r16(K, split, hash);
+    case VAR_RG: return get_kernel_rg(K, split, hash);
     case VAR_B: return get_kernel_b(K, split, hash);
     default: return get_kernel_g(K, split, hash);
     }
@@ -75,6 +77,7 @@ static MultiFn get_multi(int var, int K)
     case VAR_CL: return get_multi_cl(K);
     case VAR_N8: return get_multi_n8(K);
     case VAR_R16: return get_multi_r16(K);
+    case VAR_RG: return get_multi_rg(K);
     case VAR_B: return get_multi_b(K);
     default: return get_multi_g(K);
     }
@@ -88,6 +91,7 @@ static FixFn get_fix(int var)
     case VAR_CL: return get_fix_cl();
     case VAR_N8: return get_fix_n8();
     case VAR_R16: return get_fix_r16();
+    case VAR_RG: return get_fix_rg();
     case VAR_B: return get_fix_b();
     default: return get_fix_g();
     }
@@ -101,6 +105,7 @@ static SpecFn get_spec(int var)
     case VAR_CL: return get_spec_cl();
     case VAR_N8: return get_spec_n8();
     case VAR_R16: return get_spec_r16();
+    case VAR_RG: return get_spec_rg();
     case VAR_B: return get_spec_b();
     default: return get_spec_g();
     }
@@ -114,6 +119,7 @@ static void get_seq(int var, int K, SeqLocalFn &l, SeqWalkFn &w)
     case VAR_CL: get_seq_cl(K, l, w); break;
     case VAR_N8: get_seq_n8(K, l, w); break;
     case VAR_R16: get_seq_r16(K, l, w); break;
+    case VAR_RG: get_seq_rg(K, l, w); break;
     case VAR_B: get_seq_b(K, l, w); break;
     default: get_seq_g(K, l, w); break;
     }
@@ -138,9 +144,12 @@ struct fsm {
     bool permutation = false;  // every in-alphabet symbol permutes the states: paths never meet
     fsm_options opt{};
     // device tables
-    void *d_img[9] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
-    uint32_t img_bytes[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
+    void *d_img[10] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    uint32_t img_bytes[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     uint32_t ncls = 0, cl_magic = 0;  // CL variant
+    uint32_t rc_comp = 0;                // region counting (byte mode, accept-partitioned ids)
+    uint32_t r_logl = 0;                 // RG: log2 of the lanes sharing one table copy
+    uint32_t rc_nA = 0, cl_rc_t = 0;     // ids [0, nA) count 0 (1 if rc_comp); CL: R(nA), the row address
     // static-frequency renumbering (hot-state caching): user <-> internal ids
     bool renumbered = false;
     std::vector<uint32_t> perm, inv;
@@ -256,7 +265,7 @@ extern "C" int fsm_hot_state_order(const uint32_t *table, uint32_t n_states, uin
 
 static void free_all(fsm *f)
 {
-    for (int i = 0; i < 9; i++) cudaFree(f->d_img[i]);
+    for (int i = 0; i < 10; i++) cudaFree(f->d_img[i]);
     cudaFree(f->d_inv);
     cudaFree(f->d_lb);
     cudaFree(f->d_nimg);
@@ -322,11 +331,28 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
     f->mode = input_mode;
     build_byte_dfa(table, n_states, alphabet, accept_mask, bits, f->dfa);
     f->start_int = start;
+    // the look-back table ranks in user ids (reading A5: ties -> the smaller user id), then is
+    // mapped to the internal ids below
+    f->lb.resize(256 * KMAX);
+    f->nimg.resize(256);
+    build_lookback(f->dfa, f->lb.data(), f->nimg.data());
     if (!bits && f->dfa.n > 256 && f->dfa.n <= 32768) {
         // tables beyond shared memory: hot-state caching needs hot rows = small ids (Sec. 4.2)
         renumber_by_frequency(f->dfa, n_states, f->perm, f->inv);
         f->renumbered = true;
+    } else if (!bits && f->dfa.n <= 256) {
+        // region counting (R16, CL): accept increments become a function of the destination id
+        uint32_t nA = 0;
+        bool comp = false;
+        renumber_by_accept(f->dfa, n_states, accept_mask, f->perm, f->inv, nA, comp);
+        f->renumbered = true;
+        f->rc_nA = nA;
+        f->rc_comp = comp ? 1u : 0u;
+    }
+    if (f->renumbered) {
         f->start_int = f->perm[start];
+        for (auto &v : f->lb)
+            if (v != 0xFFFFu) v = (uint16_t)f->perm[v];
     }
     {   // paths of a DFA whose every symbol is a bijection never converge (R5 default below)
         bool perm = true;
@@ -342,9 +368,6 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         }
         f->permutation = perm;
     }
-    f->lb.resize(256 * KMAX);
-    f->nimg.resize(256);
-    build_lookback(f->dfa, f->lb.data(), f->nimg.data());
     const uint32_t n = f->dfa.n;
     // N > 256: the u32 table in L2 with the L1 acting as a hardware hot-row cache (G) measured faster
     // up to ~2K states (1027-state AC: 1.12 vs 0.98 TB/s); beyond that explicit hot-state caching in
@@ -354,7 +377,11 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
     // up to 8 accepts per byte, which N8's 1-bit count field cannot hold, so it keeps P8.
     // 8 < N <= 16: R16 (lane-replicated byte entries, conflict-free LDS.U8) measured +23..38 % over B
     // (random-bank LDS.U16): (16, 2, k=2) 2265 -> 3034, (16, 1, k=1) 2341 -> 3224 GB/s.
-    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : (n <= 8 && !bits) ? VAR_N8 : n <= 8 ? VAR_P8 : n <= 16 ? VAR_R16 : n <= 256 ? VAR_B
+    // 16 < N <= 256 in byte mode: RG (R16's layout in fewer copies, bank-conflict degree of 2^logl
+    // lanes instead of 32) measured +2..24 % over B: (24, 2) 2254 -> 2752, (32, 3) 2186 -> 2685,
+    // (64, 4) 1908 -> 2180, (255, 2) 2225 -> 2270 GB/s.
+    f->auto_variant = (n <= 4 && !bits) ? VAR_P4 : (n <= 8 && !bits) ? VAR_N8 : n <= 8 ? VAR_P8 : (n <= 16 && !bits) ? VAR_R16
+                    : (n <= 256 && !bits) ? VAR_RG : n <= 256 ? VAR_B
                     : (f->renumbered && n > 2048) ? VAR_HS : VAR_G;
     f->opt.chunk_bytes = 0;
     f->opt.threads_per_tile = 0;  // auto: max_threads(K)
@@ -384,10 +411,18 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         if ((rc = upload(&f->d_img[VAR_P8], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_P8] = 0;
     }
-    if (n <= 16) {
+    if (n <= 16 && !bits) {  // region counting: byte mode only (accept-partitioned ids)
         auto img = image_r16(f->dfa);
         if ((rc = upload(&f->d_img[VAR_R16], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_R16] = n * 8192u;  // lane-replicated in shared memory
+    }
+    if (n <= 256 && !bits) {  // RG: 32 >> logl copies of the R16 layout, <= 128 KiB (logl = 0: R16's)
+        uint32_t logl = 0;
+        while ((n << 13) >> logl > (128u << 10)) logl++;
+        auto img = image_r16(f->dfa);
+        if ((rc = upload(&f->d_img[VAR_RG], img.data(), img.size()))) return fail(rc);
+        f->img_bytes[VAR_RG] = (n * 8192u) >> logl;
+        f->r_logl = logl;
     }
     if (n <= 256) {
         auto img = image_b(f->dfa);
@@ -406,17 +441,19 @@ extern "C" int fsm_create_ex(const uint32_t *table, uint32_t n_states, uint32_t 
         if ((rc = upload(&f->d_img[VAR_HS], img.data(), img.size()))) return fail(rc);
         f->img_bytes[VAR_HS] = (uint32_t)img.size();
     }
-    {
-        // CL: byte classes + lane-replicated class-compressed table when it fits shared memory
+    if (!bits) {
+        // CL: byte classes + lane-replicated class-compressed table when it fits below the class map
+        // (u16 entries = row addresses, so the whole table must lie below shared address 0x10000)
         std::vector<uint32_t> cls, rep;
-        const uint32_t nc = cl_pad(byte_classes(f->dfa, cls, rep));
-        if (nc >= 2 && (uint64_t)f->dfa.n * nc * 128 <= kClMaxTable) {  // entry table below the class map
+        const uint32_t nc = byte_classes(f->dfa, cls, rep), rb = cl_slots(nc) * 128;
+        if (nc >= 2 && (uint64_t)f->dfa.n * rb <= kClMaxTable) {
             auto img = image_cl(f->dfa, cls, rep);
             if ((rc = upload(&f->d_img[VAR_CL], img.data(), img.size()))) return fail(rc);
-            f->img_bytes[VAR_CL] = (uint32_t)((size_t)f->dfa.n * nc * 128);
+            f->img_bytes[VAR_CL] = f->dfa.n * rb;
             f->ncls = nc;
-            f->cl_magic = (uint32_t)((((uint64_t)1 << 32) + nc - 1) / nc);
-            if (f->auto_variant == VAR_B) f->auto_variant = VAR_CL;
+            f->cl_magic = (uint32_t)((((uint64_t)1 << 32) + rb - 1) / rb);  // id = (R - 0x400) / rb
+            f->cl_rc_t = 0x400u + f->rc_nA * rb;                            // R(nA)
+            if (f->auto_variant == VAR_B || f->auto_variant == VAR_RG) f->auto_variant = VAR_CL;
         }
     }
     if (f->renumbered && (rc = upload(&f->d_inv, f->inv.data(), f->inv.size() * 4))) return fail(rc);
@@ -468,7 +505,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
-    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_R16) return FSM_EINVAL;
+    if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_RG) return FSM_EINVAL;
     if (o->variant != FSM_VARIANT_AUTO && !f->d_img[o->variant]) return FSM_EINVAL;  // too large, or retired (4)  // table too large for it
     if (o->merge > FSM_MERGE_SEQUENTIAL) return FSM_EINVAL;
     if (o->lookback_len > 1 && (o->lookback_len % 32 || o->lookback_len > 1024)) return FSM_EINVAL;
@@ -721,6 +758,9 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     p.user_out = r.user_out;
     p.ncls = f->ncls;
     p.cl_magic = f->cl_magic;
+    p.rc_t = var == VAR_CL ? f->cl_rc_t : f->rc_nA;
+    p.rc_comp = f->rc_comp;
+    p.r_logl = f->r_logl;
 
     if (var == VAR_HS) {
         // as many hot rows as fit next to this launch's scratch (227 KB per CTA)
@@ -1060,7 +1100,8 @@ extern "C" int fsm_shard_fixup(fsm_t *f, fsm_shard_t *st, uint32_t true_start, u
         fp.out = f->d_fix;
         fp.stats = f->d_stats;
         fp.kc = KConst{1u << 24, 16, 512, static_cast<const uint32_t *>(f->d_img[VAR_G]), f->hot_rows, f->ncls,
-                       f->cl_magic, 4};
+                       f->cl_magic, 4, var == VAR_CL ? f->cl_rc_t : f->rc_nA, f->rc_comp,
+                       f->r_logl};
         FixFn fn = get_fix(var);
         const size_t smem = std::max<uint32_t>(16, scratch_offset(var, f->img_bytes[var]));
         CK(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -1306,7 +1347,7 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
             if (c.k >= k_min && c.k <= k_max && (!b || c.ms < b->ms)) b = &c;
         const TuneCand best_so_far = *b;
         const int base = saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;  // what stages 1-2 ran
-        for (int v = 0; v < 9 && rc == FSM_OK; v++)
+        for (int v = 0; v < 10 && rc == FSM_OK; v++)
             if (f->d_img[v] && v != base) rc = run(best_so_far.k, best_so_far.lookback, best_so_far.eager, v);
     }
     // stage 4: R5 pre-resolution (top-1 vs every candidate) at the best setting so far

@@ -63,20 +63,11 @@ inline int build_byte_dfa(const uint32_t *table, uint32_t n_states, uint32_t alp
     return 0;
 }
 
-// Static-frequency renumbering for hot-state caching (Sec. 4.2): the frequency of a state is its
-// in-degree in the transition table (P:229, "the frequency of each of states a and c is 4");
-// states are renumbered by decreasing frequency (ties: smaller id first) so that the hottest rows
-// are the ids [0, H).  The sink (if any) keeps the last id.  perm[old] = new, inv[new] = old.
-inline void renumber_by_frequency(ByteDFA &d, uint32_t n_user, std::vector<uint32_t> &perm,
-                                  std::vector<uint32_t> &inv)
+// Renumber the states by `order` (order[new] = old for the n_user user states; the sink, if any,
+// keeps the last id): perm[old] = new, inv[new] = old.
+inline void apply_order(ByteDFA &d, uint32_t n_user, const std::vector<uint32_t> &order, std::vector<uint32_t> &perm,
+                        std::vector<uint32_t> &inv)
 {
-    std::vector<uint64_t> indeg(d.n, 0);
-    for (uint32_t s = 0; s < n_user; s++)
-        for (uint32_t c = 0; c < 256; c++) indeg[d.next[(size_t)s * 256 + c]]++;
-    std::vector<uint32_t> order(n_user);
-    for (uint32_t s = 0; s < n_user; s++) order[s] = s;
-    std::stable_sort(order.begin(), order.end(),
-                     [&](uint32_t a, uint32_t b) { return indeg[a] != indeg[b] ? indeg[a] > indeg[b] : a < b; });
     perm.assign(d.n, 0);
     inv.assign(d.n, 0);
     for (uint32_t r = 0; r < n_user; r++) {
@@ -94,6 +85,43 @@ inline void renumber_by_frequency(ByteDFA &d, uint32_t n_user, std::vector<uint3
     d.next.swap(nx);
     d.inc.swap(ic);
 }
+
+// Static-frequency renumbering for hot-state caching (Sec. 4.2): the frequency of a state is its
+// in-degree in the transition table (P:229, "the frequency of each of states a and c is 4");
+// states are renumbered by decreasing frequency (ties: smaller id first) so that the hottest rows
+// are the ids [0, H).  The sink (if any) keeps the last id.  perm[old] = new, inv[new] = old.
+inline void renumber_by_frequency(ByteDFA &d, uint32_t n_user, std::vector<uint32_t> &perm,
+                                  std::vector<uint32_t> &inv)
+{
+    std::vector<uint64_t> indeg(d.n, 0);
+    for (uint32_t s = 0; s < n_user; s++)
+        for (uint32_t c = 0; c < 256; c++) indeg[d.next[(size_t)s * 256 + c]]++;
+    std::vector<uint32_t> order(n_user);
+    for (uint32_t s = 0; s < n_user; s++) order[s] = s;
+    std::stable_sort(order.begin(), order.end(),
+                     [&](uint32_t a, uint32_t b) { return indeg[a] != indeg[b] ? indeg[a] > indeg[b] : a < b; });
+    apply_order(d, n_user, order, perm, inv);
+}
+
+// Accept-partitioned renumbering (byte mode; the region-counting variants R16 / CL):
+// the larger of F and Q \ F gets the ids [0, nA), the smaller one [nA, n_user), each in user order;
+// the sink keeps the last id.  A step's accept increment is then a function of the destination id
+// alone -- [q >= nA], or its complement when the high region is Q \ F -- which the kernels take as
+// the carry of q + 2^32 - nA, so the table entries carry the bare next state.  The sink's increment
+// is unspecified (a path that enters it ends in FSM_ESYMBOL).
+inline void renumber_by_accept(ByteDFA &d, uint32_t n_user, const uint8_t *accept, std::vector<uint32_t> &perm,
+                               std::vector<uint32_t> &inv, uint32_t &nA, bool &comp)
+{
+    std::vector<uint32_t> fin, non;
+    for (uint32_t s = 0; s < n_user; s++) ((accept && accept[s]) ? fin : non).push_back(s);
+    comp = fin.size() > non.size();
+    const std::vector<uint32_t> &lo = comp ? fin : non, &hi = comp ? non : fin;
+    nA = (uint32_t)lo.size();
+    std::vector<uint32_t> order(lo);
+    order.insert(order.end(), hi.begin(), hi.end());
+    apply_order(d, n_user, order, perm, inv);
+}
+
 
 // HS image: the first `hot` rows as u16 entries next | count << 15 (byte mode, N <= 32768).
 inline std::vector<uint8_t> image_hs(const ByteDFA &d, uint32_t hot)
@@ -128,21 +156,27 @@ inline uint32_t byte_classes(const ByteDFA &d, std::vector<uint32_t> &cls, std::
     return (uint32_t)rep.size();
 }
 
-// CL image: u32 [256] class id per byte, then u32 [N][ncls_pad] entries next * (ncls_pad * 128) | count;
-// ncls_pad = ncls rounded up to even so that the stride is a multiple of 256 and the entry's low
-// byte holds only the count (the kernel adds it with one DP4A).
-inline uint32_t cl_pad(uint32_t ncls) { return (ncls + 1) & ~1u; }
+// CL image (byte mode, accept-partitioned ids): u32 [256] class id per byte, then per state s and
+// slot q < nslot = ceil(ncls / 2) one u32 holding the u16 entries of classes 2q, 2q + 1: R(next) =
+// 0x400 + next * nslot * 128, the shared address of the next state's row (speck_kernel.cuh TableCL;
+// the kernel checks that dynamic shared memory starts at 0x400).  A padding class is never indexed.
+inline uint32_t cl_slots(uint32_t ncls) { return (ncls + 1) >> 1; }
 inline std::vector<uint8_t> image_cl(const ByteDFA &d, const std::vector<uint32_t> &cls,
                                      const std::vector<uint32_t> &rep)
 {
-    const uint32_t ncls = cl_pad((uint32_t)rep.size()), stride = ncls * 128;
-    std::vector<uint8_t> img((256 + (size_t)d.n * ncls) * 4);
+    const uint32_t nslot = cl_slots((uint32_t)rep.size()), rb = nslot * 128;
+    std::vector<uint8_t> img((256 + (size_t)d.n * nslot) * 4);
     uint32_t *p = reinterpret_cast<uint32_t *>(img.data());
     for (uint32_t c = 0; c < 256; c++) p[c] = cls[c];
     for (uint32_t s = 0; s < d.n; s++)
-        for (uint32_t k = 0; k < ncls; k++) {
-            const uint32_t r = rep[k < rep.size() ? k : 0];  // padding class: never indexed
-            p[256 + (size_t)s * ncls + k] = d.next[(size_t)s * 256 + r] * stride | d.inc[(size_t)s * 256 + r];
+        for (uint32_t q = 0; q < nslot; q++) {
+            uint32_t w = 0;
+            for (uint32_t h = 0; h < 2; h++) {
+                const uint32_t x = 2 * q + h;
+                if (x >= rep.size()) continue;
+                w |= (0x400u + d.next[(size_t)s * 256 + rep[x]] * rb) << (16 * h);
+            }
+            p[256 + (size_t)s * nslot + q] = w;
         }
     return img;
 }
@@ -198,12 +232,12 @@ inline std::vector<uint8_t> image_n8(const ByteDFA &d)
     return img;
 }
 
-// R16 (N <= 16): byte entries E[s][c] = next | count << 4, row-major (the kernel lane-replicates
-// each u32 of four entries).
+// R16 (N <= 16, byte mode): byte entries E[s][c] = next (accept-partitioned ids: the count is the
+// kernel's region test), row-major (the kernel lane-replicates each u32 of four entries).
 inline std::vector<uint8_t> image_r16(const ByteDFA &d)
 {
     std::vector<uint8_t> img((size_t)d.n * 256);
-    for (size_t i = 0; i < (size_t)d.n * 256; i++) img[i] = (uint8_t)(d.next[i] | ((uint32_t)d.inc[i] << 4));
+    for (size_t i = 0; i < (size_t)d.n * 256; i++) img[i] = (uint8_t)d.next[i];
     return img;
 }
 

@@ -2,7 +2,7 @@
 //
 // For every chunk (start byte b): the image of x[b-Lw-1] (the host look-back table) is run
 // through the Lw bytes x[b-Lw .. b) and the reached states are ranked by multiplicity (how many
-// image states reach each), ties to the smaller id; the top k + kExt distinct states are written
+// image states reach each), ties to the smaller (user) id; the top k + kExt distinct states are written
 // to spec[chunk][0 .. k + kExt) (0xFFFF = none).  Chunks whose window would reach before the start
 // of a known-start run get the single exact state; keyed runs and short prefixes fall back to the
 // depth-1 look-back.  One thread per chunk; the fused kernel then only reads its chunk's list.
@@ -71,14 +71,19 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
                 for (int j = 0; j < KMAX; j++) m += ((uint32_t)j < ni && y[j] == y[i]) ? 1u : 0u;
                 mult[i] = (uint32_t)i < ni ? m : 0u;
             }
-            // selection: repeatedly take the best remaining (multiplicity desc, id asc)
+            // ties go to the smaller USER id (as in the host look-back table, reading A5)
+            uint32_t uy[KMAX];
+#pragma unroll
+            for (int i = 0; i < KMAX; i++) uy[i] = p.inv ? __ldg(p.inv + y[i]) : y[i];
+            // selection: repeatedly take the best remaining (multiplicity desc, user id asc)
             for (; written < stride; written++) {
-                uint32_t bm = 0, bs = NOSTATE;
+                uint32_t bm = 0, bs = NOSTATE, bu = 0xFFFFFFFFu;
 #pragma unroll
                 for (int i = 0; i < KMAX; i++)
-                    if (mult[i] > bm || (mult[i] == bm && mult[i] && y[i] < bs)) {
+                    if (mult[i] > bm || (mult[i] == bm && mult[i] && uy[i] < bu)) {
                         bm = mult[i];
                         bs = y[i];
+                        bu = uy[i];
                     }
                 if (!bm) break;
 #pragma unroll

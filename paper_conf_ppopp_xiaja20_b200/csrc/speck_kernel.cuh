@@ -27,7 +27,7 @@
 
 namespace speck {
 
-enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, /* 4: retired (H8) */ VAR_HS = 5, VAR_CL = 6, VAR_N8 = 7, VAR_R16 = 8 };
+enum { VAR_P4 = 0, VAR_P8 = 1, VAR_B = 2, VAR_G = 3, /* 4: retired (H8) */ VAR_HS = 5, VAR_CL = 6, VAR_N8 = 7, VAR_R16 = 8, VAR_RG = 9 };
 constexpr int kThreads = 256;  // auxiliary kernels
 // Eager completion (NEXT-3): per chunk, up to kExt image states beyond the speculated ones are run
 // in lockstep over the chunk's first kExtWindow bytes; entry = key | slot << 16 | (delta & 0xFFF) << 20.
@@ -119,11 +119,26 @@ __device__ __forceinline__ uint32_t lds_u8(uint32_t a)
     asm("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
     return v;
 }
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a)
+{
+    uint32_t v;
+    asm("ld.shared.u16 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
 __device__ __forceinline__ uint2 lds_v2(uint32_t a)
 {
     uint2 v;
     asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
     return v;
+}
+// acc + [x >= T] with negT = 2^32 - T: the carry out of x + negT, added by a second add (IADD3 and
+// IADD3.X, each issued on either integer pipe at full rate; measured tools/pipe_probe: IMAD.HI takes
+// 4 cycles per warp per SMSP, an add 1).  The region count of R16 / RG / CL.
+__device__ __forceinline__ uint32_t add_ge(uint32_t acc, uint32_t x, uint32_t negT)
+{
+    uint32_t d;
+    asm("{\n\t.reg .u32 t;\n\tadd.cc.u32 t, %1, %2;\n\taddc.u32 %0, %3, 0;\n\t}" : "=r"(d) : "r"(x), "r"(negT), "r"(acc));
+    return d;
 }
 __device__ __forceinline__ uint32_t dp4a_u(uint32_t a, uint32_t b, uint32_t c)
 {
@@ -134,18 +149,19 @@ __device__ __forceinline__ uint32_t dp4a_u(uint32_t a, uint32_t b, uint32_t c)
 constexpr uint32_t kPackedBase = 0x10000u;  // shared-window address of the packed tables
 constexpr uint32_t kSmemWindowBase = 1024u;  // dynamic shared memory starts here (measured: tools/smem_probe)
 __host__ __device__ constexpr bool is_packed(int var) { return var == 0 || var == 1 || var == 7; }
-// CL: the entry table sits at the start of dynamic smem (shared address 0x400 up to < 0x20000) and
-// the 32 KiB lane-replicated class map at the fixed shared address 0x20000, so a class-map address
-// is (byte << 7) | lane * 4 | 0x20000 -- disjoint bit fields, one LOP3 after the byte's shift.
-constexpr uint32_t kClMapBase = 0x20000u;
+// CL: the entry table sits at the start of dynamic smem (shared addresses [0x400, 0x10000): its u16
+// entries are shared addresses) and the lane-replicated class map at the fixed shared address
+// 0x10000 with a 256-byte stride, so a class-map address is ONE PRMT of the input word
+// (0x10000 | byte << 8 | lane * 4, the packed tables' form).
+constexpr uint32_t kClMapBase = 0x10000u;
 constexpr uint32_t kClMaxTable = kClMapBase - 1024u;  // entry-table bytes that fit below the map
 // Offset (from the start of dynamic smem) of the scratch area that follows the table.  Packed
-// tables occupy the window [0x10000, 0x20000); CL's class map [0x20000, 0x28000); everything else
-// goes above the table.
+// tables and CL's class map occupy the window [0x10000, 0x20000); everything else goes above the
+// table.
 __host__ __device__ constexpr uint32_t scratch_offset(int var, uint32_t table_bytes)
 {
     return is_packed(var) ? (kPackedBase + 65536u - kSmemWindowBase)
-         : var == 6 ? (kClMapBase + 256u * 128u - kSmemWindowBase)
+         : var == 6 ? (kClMapBase + 256u * 256u - kSmemWindowBase)
          : ((table_bytes + 15u) & ~15u);
 }
 __device__ __forceinline__ void check_smem_window(int var, uint32_t need)
@@ -164,10 +180,12 @@ struct KConst {
     uint32_t hot_rows;     // HS: states [0, hot_rows) have their rows in shared memory
     uint32_t ncls, cl_magic;  // CL: byte classes, ceil(2^32 / ncls)
     uint32_t k_4;             // N8
+    uint32_t rc_t, rc_comp;      // region counting (R16, RG, CL; Params)
+    uint32_t r_logl;             // RG: log2 of the lanes sharing a table copy
 };
 __device__ __forceinline__ KConst kconst(const Params &p)
 {
-    return KConst{p.k_1e24, p.k_16, p.k_512, p.table_g, p.hot_rows, p.ncls, p.cl_magic, p.k_4};
+    return KConst{p.k_1e24, p.k_16, p.k_512, p.table_g, p.hot_rows, p.ncls, p.cl_magic, p.k_4, p.rc_t, p.rc_comp, p.r_logl};
 }
 
 // ------------------------------------------------------------------- table-placement variants --
@@ -193,12 +211,9 @@ struct TablePacked {
     static constexpr bool kWide = VAR == VAR_P8;
     static constexpr uint32_t kX = 0x4544u;
     uint32_t lanereg;
-    uint32_t c24, c16;  // 1 << 24 and 16 from kernel params so that ptxas keeps IMAD / IMAD.HI (FMA pipe)
     __device__ __forceinline__ void setup(uint8_t *, const void *g, uint32_t, const KConst &kc)
     {
         lanereg = kPackedBase | ((threadIdx.x & 31) * (kWide ? 8 : 4));
-        c24 = kc.k_1e24;
-        c16 = kc.k_16;
         if (kWide) {
             const uint2 *rows = static_cast<const uint2 *>(g);
             for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
@@ -215,7 +230,7 @@ struct TablePacked {
     }
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return kWide ? st : (st | 0x44444440u); }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur & 0xFu; }
-    // P8: acc = count * 16 (ALU accumulation) + accf (FMA accumulation).
+    // P8: acc = count * 16.
     // P4: acc = sum of (0x44 + lagged count) over n steps; the last step's count sits in cur.
     __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t cur, uint64_t n) const
     {
@@ -232,9 +247,8 @@ struct TablePacked {
             const uint2 r = lds_v2(a);
 #pragma unroll
             for (int s = 0; s < K; s++) {
-                cur[s] = prmt(r.x, r.y, cur[s]);                       // the chain: one PRMT per step
-                if (((j + s) & 1) == 0) acc[s] += cur[s] & 0xF0u;      // ALU: LOP3 (+ half an IADD3)
-                else accf[s] = mad_hi(cur[s] * c24, c16, accf[s]);     // FMA: IMAD, IMAD.HI (field >> 4)
+                cur[s] = prmt(r.x, r.y, cur[s]);  // the chain: one PRMT per step
+                acc[s] += cur[s] & 0xF0u;         // LOP3 + IADD3 (an IMAD.HI would take 4 cycles per warp)
             }
         } else {
             const uint32_t r = lds_u32(a);
@@ -348,15 +362,15 @@ struct TableB {
     {
         sm = s;
         c512 = kc.k_512;
-        c2e24 = kc.k_1e24;
         const uint4 *src = static_cast<const uint4 *>(g);
         uint4 *dst = reinterpret_cast<uint4 *>(s);
         for (uint32_t i = threadIdx.x; i < n * 32; i += blockDim.x) dst[i] = __ldg(src + i);
     }
-    uint32_t c512, c2e24;
+    uint32_t c512;
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
+    // acc counts in units of 256 (at most 8 x 8 KiB x 256 = 2^24 per chunk)
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return (acc >> 8) + accf; }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                          uint32_t (&accf)[K]) const
@@ -368,7 +382,7 @@ struct TableB {
             // entry = next | count << 8; address = next * 512 + 2c on the FMA pipe (IMAD)
             const uint32_t e = *reinterpret_cast<const uint16_t *>(base + mad_lo(cur[s], c512, 0u));
             cur[s] = e & 0xFFu;
-            accf[s] = mad_hi(e, c2e24, accf[s]);  // + (e >> 8), FMA pipe
+            acc[s] = acc[s] + e - cur[s];  // + 256 * count: one IADD3 (IMAD.HI takes 4 cycles per warp)
         }
     }
     using Row = uint32_t;
@@ -456,113 +470,129 @@ struct TableHS {
     __device__ __forceinline__ uint32_t apply(Row c, uint32_t st, uint32_t &cnt) const { return lookup(st, c, cnt); }
 };
 
-// CL: byte-class compressed, lane-replicated table (DFAs with few distinct byte columns, e.g. the
-// HTML tokenizer: 38 states x 24 classes).  Entry table: u32 [N][ncls][32 lanes] at the start of
-// dynamic smem, entry = next * stride | count (stride = ncls * 128, count in bits 0-3).  Class map:
-// u32 [256][32 lanes] at shared address 0x20000 = shared address of the lane's copy of the class
-// row.  Every lookup is conflict-free (each lane reads its own bank); the class-map address of
-// byte j of a word is one shift + one LOP3 ((x & 0x7F80) | 0x20000 | lane * 4), off the chain; the
-// chain step is LOP3 + IADD + LDS.32 with the count taken by one DP4A of the entry's low byte.
-// Chains carry the entry itself (next * stride | count); ids are recovered by a multiply-high.
+// CL: byte-class compressed, lane-replicated table (byte-mode DFAs with few distinct byte columns,
+// e.g. the HTML tokenizer: 38 states x 24 classes).  Row of state s at R(s) = 0x400 + s * RB
+// (RB = ceil(ncls / 2) * 128): the u16 entry (s, class x) of lane l sits at
+//   R(s) + (x >> 1) * 128 + l * 4 + (x & 1) * 2
+// and holds R(next) -- the chain value IS the next row's address.  Class map: u32 [256][32 lanes]
+// at 0x10000 + byte * 256 + lane * 4 = the lane's offset of the byte's class, (x >> 1) * 128 + l * 4
+// + (x & 1) * 2.  Every lookup is conflict-free (each lane reads its own bank).  Per byte: PRMT
+// (class-map address) + LDS (class offset), off the chain; IADD + LDS.U16 on the chain; two adds for
+// the count (region counting on the row address: ids are accept-partitioned, so [next >= nA] =
+// [R(next) >= R(nA)] = the carry of R(next) + 2^32 - R(nA)).  Ids are recovered by a multiply-high.
 struct TableCL {
     uint32_t cmreg;   // kClMapBase | lane * 4
-    uint32_t stride, magic;
+    uint32_t tbase, rb, idmagic, negT, comp;
     __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n, const KConst &kc)
     {
-        const uint32_t tbase = (uint32_t)__cvta_generic_to_shared(s);  // 0x400 (checked)
-        const uint32_t ncls = kc.ncls;
-        stride = ncls * 128u;
-        magic = kc.cl_magic;
+        tbase = (uint32_t)__cvta_generic_to_shared(s);  // 0x400 (checked)
+        const uint32_t nslot = (kc.ncls + 1) >> 1;
+        rb = nslot * 128u;
+        idmagic = kc.cl_magic;
+        negT = 0u - kc.rc_t;
+        comp = kc.rc_comp;
         const uint32_t lane = threadIdx.x & 31;
         cmreg = kClMapBase | (lane * 4);
         const uint32_t *img = static_cast<const uint32_t *>(g);
         for (uint32_t i = threadIdx.x; i < 256 * 32; i += blockDim.x) {
-            const uint32_t c = i >> 5, l = i & 31;
-            const uint32_t v = tbase + __ldg(img + c) * 128u + l * 4u;  // image: class id per byte
-            asm volatile("st.shared.u32 [%0], %1;" ::"r"(kClMapBase + c * 128 + l * 4), "r"(v));
+            const uint32_t c = i >> 5, l = i & 31, x = __ldg(img + c);  // image: class id per byte
+            const uint32_t v = (x >> 1) * 128u + l * 4u + (x & 1u) * 2u;
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(kClMapBase + c * 256 + l * 4), "r"(v));
         }
-        for (uint32_t i = threadIdx.x; i < n * ncls * 32; i += blockDim.x) {
-            const uint32_t e = i >> 5, l = i & 31;
+        for (uint32_t i = threadIdx.x; i < n * nslot * 32; i += blockDim.x) {
+            const uint32_t e = i >> 5, l = i & 31;  // e = s * nslot + slot: two u16 entries
             asm volatile("st.shared.u32 [%0], %1;" ::"r"(tbase + e * 128 + l * 4), "r"(__ldg(img + 256 + e)));
         }
     }
-    __device__ __forceinline__ uint32_t init(uint32_t st) const { return st * stride; }
-    __device__ __forceinline__ uint32_t id_of(uint32_t cur) const { return __umulhi((cur & ~0xFu) >> 7, magic); }
+    __device__ __forceinline__ uint32_t init(uint32_t st) const { return tbase + st * rb; }
+    __device__ __forceinline__ uint32_t id_of(uint32_t cur) const { return __umulhi(cur - tbase, idmagic); }
     __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return id_of(cur); }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t) const { return acc + accf; }
-    // class-map address of byte j of w: the byte moved to bits 7..14, then one LOP3
-    __device__ __forceinline__ uint32_t cmaddr(uint32_t w, int j) const
+    // acc: steps into the high region, n steps in all
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t n) const
     {
-        const uint32_t x = j == 0 ? (w << 7) : (w >> (8 * j - 7));
-        return (x & 0x7F80u) | cmreg;
+        return comp ? (uint32_t)n - (acc + accf) : acc + accf;
     }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
                                          uint32_t (&accf)[K]) const
     {
-        const uint32_t cm = lds_u32(cmaddr(w, j));  // class row of this lane (off the chain)
+        const uint32_t cm = lds_u32(prmt(w, cmreg, 0x7604u | (uint32_t(j) << 4)));  // off the chain
 #pragma unroll
         for (int s = 0; s < K; s++) {
-            const uint32_t e = lds_u32((cur[s] & ~0xFu) + cm);
-            acc[s] = dp4a_u(e, 1u, acc[s]);
-            cur[s] = e;
+            cur[s] = lds_u16(cur[s] + cm);              // R(next)
+            accf[s] = add_ge(accf[s], cur[s], negT);    // + [R(next) >= R(nA)]
         }
     }
     using Row = uint32_t;
-    __device__ __forceinline__ Row row(uint32_t c) const { return lds_u32(cmreg + (c << 7)); }
+    __device__ __forceinline__ Row row(uint32_t c) const { return lds_u32(cmreg + (c << 8)); }
+    // one step in the chain representation (row address), exact count: the lockstep loops
+    __device__ __forceinline__ uint32_t step1(Row cm, uint32_t cur, uint32_t &cnt) const
+    {
+        const uint32_t e = lds_u16(cur + cm);
+        cnt += (uint32_t)(e >= 0u - negT) ^ comp;  // the accept increment (garbage only for the sink)
+        return e;
+    }
     __device__ __forceinline__ uint32_t apply(Row cm, uint32_t st, uint32_t &cnt) const
     {
-        const uint32_t e = lds_u32(st * stride + cm);
-        cnt += e & 0xFu;
-        return id_of(e);
+        return id_of(step1(cm, init(st), cnt));
     }
 };
 
-// R16: N <= 16, lane-replicated byte entries E[s][c] = next | count << 4 (count 0/1 in byte mode,
-// 0..8 in bit mode).  Lane l owns bank l: the entry (s, c) of lane l sits at shared address
+// R16: N <= 16, byte mode, lane-replicated byte entries E[s][c] = next (accept-partitioned ids,
+// region counting).  Lane l owns bank l: the entry (s, c) of lane l sits at shared address
 //   tbase + s * 8192 + (c >> 2) * 128 + l * 4 + (c & 3)
 // (the four entries of symbols 4q..4q+3 share the lane's word), so every LDS.U8 of a warp is one
 // conflict-free wavefront whatever the lanes' states and symbols -- B's u16 table at N = 16 is read at
 // random banks (72 % replays).  128 KiB at N = 16.  The symbol part of the address is computed, not
-// loaded (two LOP3 per word, two PRMT + one IMAD per byte, off the chain); the chain step is
-// LOP3 (state bits) + IMAD (row offset) + LDS.U8.  The count of an entry is taken one step late,
-// when its state bits are masked anyway: acc += cur - (cur & 0xF) = 16 * count (one IADD3); the
-// last entry's count is still in cur when count_of runs.
-struct TableR16 {
-    uint32_t lane4;   // lane * 4 in every byte
+// loaded (two LOP3 per word, two PRMT + one IMAD/LEA per byte, off the chain).  The chain step is
+// IMAD (row offset of the bare next state) + LDS.U8, and the count is two adds off the chain (region
+// counting: [q >= nA] = the carry of q + 2^32 - nA, host_tables.h renumber_by_accept) -- no ALU-only
+// operation on the chain, none for the count.
+// RG (GROUPED, N <= 256, auto for 16 < N): the same with G = 32 >> logl copies instead of 32 -- lanes
+// 2^logl * g .. 2^logl * (g + 1) - 1 share copy g, which occupies banks of their own, so a warp's
+// LDS.U8 costs the worst bank load of 2^logl lanes on 2^logl banks instead of 32 lanes on 32 (B):
+//   tbase + s * (8192 >> logl) + (c >> b) * 128 + g * 2^b + (c & (2^b - 1)),   b = 2 + logl,
+// G * N * 256 <= 128 KiB (logl = 1: N <= 32, 2: N <= 64, ...).  logl is a run-time parameter.
+template <bool GROUPED>
+struct TableRep {
+    uint32_t lane4;   // the lane's copy offset g * 2^b in every byte
     uint32_t tb;      // shared address of the table (low byte 0; PRMT source of bytes 1..3)
-    uint32_t c8192, c32;
+    uint32_t mlo;     // 2^b - 1 in every byte
+    uint32_t sstride, cmul, negT, comp;
     __device__ __forceinline__ void setup(uint8_t *s, const void *g, uint32_t n, const KConst &kc)
     {
         tb = (uint32_t)__cvta_generic_to_shared(s);
         if (tb & 0xFFu) __trap();  // the PRMT address form needs a 256-aligned table
-        lane4 = (threadIdx.x & 31) * 4u * 0x01010101u;
-        c8192 = kc.k_512 << 4;
-        c32 = kc.k_16 << 1;
-        const uint32_t *img = static_cast<const uint32_t *>(g);  // u32 [n][64]: entries 4q..4q+3 of row s
-        for (uint32_t i = threadIdx.x; i < n * 64 * 32; i += blockDim.x)
-            asm volatile("st.shared.u32 [%0], %1;" ::"r"(tb + i * 4), "r"(__ldg(img + (i >> 5))));
+        const uint32_t logl = GROUPED ? kc.r_logl : 0u, lane = threadIdx.x & 31;
+        lane4 = ((lane >> logl) << (2 + logl)) * 0x01010101u;
+        mlo = ((4u << logl) - 1u) * 0x01010101u;
+        sstride = (kc.k_512 << 4) >> logl;
+        cmul = (kc.k_16 << 1) >> logl;
+        negT = 0u - kc.rc_t;
+        comp = kc.rc_comp;
+        // smem word i: line i >> 5, copy (i & 31) >> logl, word (line << logl) | (i & (2^logl - 1))
+        // of the row-major image (u32 [n][64]: entries 4q..4q+3 of row s)
+        const uint32_t *img = static_cast<const uint32_t *>(g);
+        const uint32_t lm = (1u << logl) - 1u;
+        for (uint32_t i = threadIdx.x; i < ((n * 64 * 32) >> logl); i += blockDim.x)
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(tb + i * 4),
+                         "r"(__ldg(img + (((i >> 5) << logl) | (i & lm)))));
     }
     __device__ __forceinline__ uint32_t init(uint32_t st) const { return st; }
-    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur & 0xFu; }
-    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t cur, uint64_t) const
+    __device__ __forceinline__ uint32_t state_of(uint32_t cur) const { return cur; }
+    // acc: steps into the high region, n steps in all
+    __device__ __forceinline__ uint32_t count_of(uint32_t acc, uint32_t accf, uint32_t, uint64_t n) const
     {
-        return (acc >> 4) + (cur >> 4) + accf;
+        return comp ? (uint32_t)n - (acc + accf) : acc + accf;
     }
-    // Move the pending (one-step-late) count of the last entry into the accumulator.  Needed before
-    // the convergence collapse replaces every slot's chain by slot 0's: in bit mode the pending count
-    // (F-visits of the last widened byte) depends on the slot's own source state, not only on the
-    // common destination.
-    __device__ __forceinline__ void settle(uint32_t &cur, uint32_t &acc) const
-    {
-        acc += cur & ~0xFu;
-        cur &= 0xFu;
-    }
-    // symbol part of the address of byte j of w
+    // symbol part of the address of byte j of w.  The chain and the count are on the FMA pipe, so
+    // R16's odd bytes combine the two halves with a shift-add (LEA, ALU pipe) instead of an IMAD.
     __device__ __forceinline__ uint32_t sym(uint32_t w, int j) const
     {
-        const uint32_t lo = (w & 0x03030303u) | lane4, hi = w & 0xFCFCFCFCu;
-        return mad_lo(prmt(hi, 0u, 0x4440u | uint32_t(j)), c32, prmt(lo, tb, 0x7650u | uint32_t(j)));
+        const uint32_t m = GROUPED ? mlo : 0x03030303u;
+        const uint32_t lo = (w & m) | lane4, hi = w & ~m;
+        const uint32_t h = prmt(hi, 0u, 0x4440u | uint32_t(j)), l = prmt(lo, tb, 0x7650u | uint32_t(j));
+        return (!GROUPED && (j & 1)) ? (h << 5) + l : mad_lo(h, cmul, l);
     }
     template <int K>
     __device__ __forceinline__ void step(uint32_t w, int j, uint32_t (&cur)[K], uint32_t (&acc)[K],
@@ -571,20 +601,21 @@ struct TableR16 {
         const uint32_t a = sym(w, j);
 #pragma unroll
         for (int s = 0; s < K; s++) {
-            const uint32_t m = cur[s] & 0xFu;
-            acc[s] = acc[s] + cur[s] - m;          // 16 * count of the previous entry
-            cur[s] = lds_u8(mad_lo(m, c8192, a));  // next | count << 4
+            cur[s] = lds_u8(mad_lo(cur[s], sstride, a));  // next state
+            accf[s] = add_ge(accf[s], cur[s], negT);      // + [next >= nA]
         }
     }
     using Row = uint32_t;
     __device__ __forceinline__ Row row(uint32_t c) const { return sym(c, 0); }
     __device__ __forceinline__ uint32_t apply(Row a, uint32_t st, uint32_t &cnt) const
     {
-        const uint32_t e = lds_u8(a + st * 8192u);
-        cnt += e >> 4;
-        return e & 0xFu;
+        const uint32_t e = lds_u8(a + st * sstride);
+        cnt += (uint32_t)(e >= 0u - negT) ^ comp;  // the accept increment (garbage only for the sink)
+        return e;
     }
 };
+using TableR16 = TableRep<false>;
+using TableRG = TableRep<true>;
 
 template <int VAR> struct TableFor;
 template <> struct TableFor<VAR_P4> { using type = TablePacked<VAR_P4>; };
@@ -595,14 +626,27 @@ template <> struct TableFor<VAR_HS> { using type = TableHS; };
 template <> struct TableFor<VAR_CL> { using type = TableCL; };
 template <> struct TableFor<VAR_N8> { using type = TableN8; };
 template <> struct TableFor<VAR_R16> { using type = TableR16; };
+template <> struct TableFor<VAR_RG> { using type = TableRG; };
 
 // --------------------------------------------------------------------- a4: local processing --
 template <class TB> struct TableHasStep4 { static constexpr bool value = false; };
-// Tables whose chain value carries a count not yet added to the accumulator (R16) settle it before
-// the convergence collapse.  P4 also lags its count, but only in byte mode, where the count of an
-// entry is that of its destination state and so equal in every converged slot.
-template <class TB> struct TableHasSettle { static constexpr bool value = false; };
-template <> struct TableHasSettle<TableR16> { static constexpr bool value = true; };
+// Tables whose chain representation is not the state id but can be stepped one byte at a time
+// with an exact count (step1): the lockstep loops run in that representation (equality of two
+// chain values is equality of states) and skip the id conversions of apply().
+template <class TB> struct TableHasStep1 { static constexpr bool value = false; };
+template <> struct TableHasStep1<TableCL> { static constexpr bool value = true; };
+template <class TB>
+__device__ __forceinline__ uint32_t nat_init(const TB &tb, uint32_t st)
+{
+    if constexpr (TableHasStep1<TB>::value) return tb.init(st);
+    else return st;
+}
+template <class TB>
+__device__ __forceinline__ uint32_t nat_apply(const TB &tb, const typename TB::Row &r, uint32_t x, uint32_t &cnt)
+{
+    if constexpr (TableHasStep1<TB>::value) return tb.step1(r, x, cnt);
+    else return tb.apply(r, x, cnt);
+}
 template <> struct TableHasStep4<TableN8> { static constexpr bool value = true; };
 
 template <int K, class TB>
@@ -722,10 +766,6 @@ __device__ __forceinline__ void local_phase(const TB &tb, const uint8_t *__restr
     }
     if constexpr (K > 1) {
         if (single) {
-            if constexpr (TableHasSettle<TB>::value) {
-#pragma unroll
-                for (int s = 0; s < K; s++) tb.settle(cur[s], acc[s]);
-            }
             uint32_t c1[1] = {cur[0]}, a1[1] = {0u}, f1[1] = {0u};
             run_blocks<1, false>(tb, p, i, nblk, x0, x1, c1, a1, f1);
             for (uint64_t t = nblk << 5; t < n; t++) tb.template step<1>(__ldg(p + t), 0, c1, a1, f1);
@@ -1027,7 +1067,7 @@ __device__ __forceinline__ void named_arrive(uint32_t id, uint32_t n)
 // memory (large-K CL kernels next to a 150 KiB table do not).
 __host__ __device__ constexpr bool split_kernel(int var, int K)
 {
-    return var == 6 /* CL */ || ((var == 0 || var == 1 || var == 2 || var == 7 || var == 8) /* P4 P8 B N8 R16 */ && K >= 2);
+    return var == 6 /* CL */ || ((var == 0 || var == 1 || var == 2 || var == 7 || var == 8 || var == 9) /* P4 P8 B N8 R16 RG */ && K >= 2);
 }
 
 // Per-tile context used by re-execution and the epilogue.
@@ -1099,21 +1139,22 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
         for (int l = 0; l < K; l++) {
             const uint32_t sv = t.Sj[c * K + l];
             pres[l] = sv != 0xFFFFu;
-            y[l] = pres[l] ? sv : 0u;
+            y[l] = nat_init(tb, pres[l] ? sv : 0u);
             cy[l] = 0;
         }
         uint32_t cx = 0, cyc = 0;
         int conv = -1;
         uint64_t pos = b;
         const uint64_t wend = min(e, b + kLockstepWindow);
+        uint32_t sn = nat_init(tb, st);  // the re-executed path in the chain representation
         auto one = [&](uint32_t byte) {
             const typename TB::Row r = tb.row(byte);
-            st = tb.apply(r, st, cx);
+            sn = nat_apply(tb, r, sn, cx);
 #pragma unroll
-            for (int l = 0; l < K; l++) y[l] = tb.apply(r, y[l], cy[l]);
+            for (int l = 0; l < K; l++) y[l] = nat_apply(tb, r, y[l], cy[l]);
 #pragma unroll
             for (int l = 0; l < K; l++)
-                if (pres[l] && conv < 0 && y[l] == st) {
+                if (pres[l] && conv < 0 && y[l] == sn) {
                     conv = l;
                     cyc = cy[l];
                 }
@@ -1150,16 +1191,18 @@ __device__ void resolve(const TB &tb, const TileCtx &t, uint32_t st, uint32_t c,
         }
         if (conv < 0 && pos < e) {  // past the lockstep window: the re-executed path alone
             if (t.aligned) {
-                for (; (pos & 15) && pos < e; pos++) st = tb.apply(tb.row(__ldg(t.in + pos)), st, cx);
+                for (; (pos & 15) && pos < e; pos++) sn = nat_apply(tb, tb.row(__ldg(t.in + pos)), sn, cx);
                 for (; pos + 16 <= e; pos += 16) {
                     const uint4 v = ldg128(t.in + pos);
                     const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-                    for (int q = 0; q < 16; q++) st = tb.apply(tb.row((w4[q >> 2] >> (8 * (q & 3))) & 0xFFu), st, cx);
+                    for (int q = 0; q < 16; q++) sn = nat_apply(tb, tb.row((w4[q >> 2] >> (8 * (q & 3))) & 0xFFu), sn, cx);
                 }
             }
-            for (; pos < e; pos++) st = tb.apply(tb.row(__ldg(t.in + pos)), st, cx);
+            for (; pos < e; pos++) sn = nat_apply(tb, tb.row(__ldg(t.in + pos)), sn, cx);
         }
+        if constexpr (TableHasStep1<TB>::value) st = tb.state_of(sn);
+        else st = sn;
         chain = c == last_c + 1 ? chain + 1 : 1;
         last_c = c;
         rc.chunks++;
@@ -1619,14 +1662,14 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
                 bool live[kExt];
 #pragma unroll
                 for (int l = 0; l < K; l++) {
-                    y[l] = S[l] == NOSTATE ? 0u : S[l];
+                    y[l] = nat_init(tb, S[l] == NOSTATE ? 0u : S[l]);
                     cy[l] = 0;
                 }
                 int nlive = 0;
 #pragma unroll
                 for (int q = 0; q < kExt; q++) {
                     live[q] = Xc[q] != NOSTATE;
-                    u[q] = live[q] ? Xc[q] : 0u;
+                    u[q] = nat_init(tb, live[q] ? Xc[q] : 0u);
                     cu[q] = 0;
                     nlive += live[q];
                 }
@@ -1646,11 +1689,11 @@ __device__ __forceinline__ void speck_body(const Params &p0, const Params *__res
                         const uint32_t byte = (xb.w[pos >> 2] >> (8 * (pos & 3))) & 0xFFu;
                         const typename TB::Row r = tb.row(byte);
 #pragma unroll
-                        for (int l = 0; l < K; l++) y[l] = tb.apply(r, y[l], cy[l]);
+                        for (int l = 0; l < K; l++) y[l] = nat_apply(tb, r, y[l], cy[l]);
 #pragma unroll
                         for (int q = 0; q < kExt; q++) {
                             if (!live[q]) continue;
-                            u[q] = tb.apply(r, u[q], cu[q]);
+                            u[q] = nat_apply(tb, r, u[q], cu[q]);
 #pragma unroll
                             for (int l = 0; l < K; l++)
                                 if (live[q] && S[l] != NOSTATE && y[l] == u[q]) {

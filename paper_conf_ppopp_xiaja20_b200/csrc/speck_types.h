@@ -105,13 +105,19 @@ struct Params {
     const uint32_t *table_g;       // full u32 table (HS variant's cold rows)
     uint32_t hot_rows;             // HS variant: rows cached in shared memory
     const uint32_t *inv;           // internal -> user state ids (renumbered handles), or null
-    uint32_t ncls, cl_magic;       // CL variant: byte classes and ceil(2^32 / ncls)
+    uint32_t ncls, cl_magic;       // CL variant: byte classes and ceil(2^32 / row bytes) (state ids)
     uint32_t *user_out;            // optional: the last tile also writes {user state, 0, count lo, hi} here
     uint32_t eager_window;         // NEXT-3 eager completion: bytes of lockstep per chunk (0 = off)
     uint32_t k_4;                  // N8 variant: FMA-pipe constant 4, see k_1e24 above
     uint32_t preresolve;           // R5: tile-start slots (in rank order) resolved before publishing A
     uint32_t spec_all;             // test hook: `spec` also overrides chunk 0 of a known-start run
     uint4 *dbg;                    // test hook: warp-scan levels of tile 0, warp 0 ([6][32][KMAX]), or null
+    // region counting (byte mode, accept-partitioned ids, host_tables.h renumber_by_accept): the
+    // accept increment of a step into state q is [q >= nA] (R16, RG: rc_t = nA) or [R(q) >= R(nA)]
+    // (CL's row addresses: rc_t = R(nA)); rc_comp: the high region is the NON-accepting one
+    // (count = steps - that).
+    uint32_t rc_t, rc_comp;
+    uint32_t r_logl;               // RG variant: log2 of the lanes that share one table copy
 };
 
 }  // namespace speck

@@ -18,8 +18,8 @@ FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_EUNSUPPORTED = 0, -1
 FSM_INPUT_BYTES, FSM_INPUT_BITS_MSB = 0, 1
 FSM_KMAX = 16
 FSM_VARIANT_AUTO, FSM_VARIANT_P4, FSM_VARIANT_P8, FSM_VARIANT_B, FSM_VARIANT_G = -1, 0, 1, 2, 3
-FSM_VARIANT_HS, FSM_VARIANT_CL, FSM_VARIANT_N8, FSM_VARIANT_R16 = 5, 6, 7, 8
-VARIANT_NAMES = {0: "P4", 1: "P8", 2: "B", 3: "G", 5: "HS", 6: "CL", 7: "N8", 8: "R16"}
+FSM_VARIANT_HS, FSM_VARIANT_CL, FSM_VARIANT_N8, FSM_VARIANT_R16, FSM_VARIANT_RG = 5, 6, 7, 8, 9
+VARIANT_NAMES = {0: "P4", 1: "P8", 2: "B", 3: "G", 5: "HS", 6: "CL", 7: "N8", 8: "R16", 9: "RG"}
 FSM_MERGE_PARALLEL, FSM_MERGE_SEQUENTIAL = 0, 1
 FSM_EAGER_OFF = 1
 FSM_PRERESOLVE_NONE = 0x80000000

@@ -132,7 +132,7 @@ def test_map_compose_vs_model_random(seed):
 
 def test_variant_enum_matches_header():
     """The binding's variant ids and names are the header's FSM_VARIANT_* enum (one table variant
-    per id; R16 = 8 is the newest)."""
+    per id; RG = 9 is the newest)."""
     txt = open(os.path.join(ROOT, "include", "fsmspec.h")).read()
     txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
     enum = {m.group(1): int(m.group(2)) for m in re.finditer(r"FSM_VARIANT_([A-Z0-9]+)\s*=\s*(-?\d+)", txt)}

@@ -35,15 +35,18 @@ def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
     return res, st
 
 
-VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8, "RG": 9}
 
 
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
+    # R16 and CL use region counting (accept-partitioned ids): byte mode only
     return {"P4": n <= 4 and not dfa.bit_mode, "P8": n <= 8,
-            "N8": n <= 8 and not dfa.bit_mode, "R16": n <= 16,
+            "N8": n <= 8 and not dfa.bit_mode, "R16": n <= 16 and not dfa.bit_mode,
+            "RG": n <= 256 and not dfa.bit_mode,
             "B": n <= 256, "G": True, "HS": not dfa.bit_mode and n <= 32768,
-            "CL": _n_classes(dfa) >= 2 and n * ((_n_classes(dfa) + 1) & ~1) * 128 <= 0x20000 - 1024}[var]
+            "CL": not dfa.bit_mode and _n_classes(dfa) >= 2
+            and n * ((_n_classes(dfa) + 1) // 2) * 128 <= 0x10000 - 1024}[var]
 
 
 def _n_classes(dfa):
@@ -92,7 +95,8 @@ def test_c_comment_text(var, chunk):
 
 
 # --------------------------------------------------------------------- random DFAs, all variants, all k
-CASES = [(2, 2), (4, 2), (4, 4), (7, 3), (8, 1), (8, 2), (8, 8), (16, 2), (16, 5), (100, 4), (255, 8),
+CASES = [(2, 2), (4, 2), (4, 4), (7, 3), (8, 1), (8, 2), (8, 8), (16, 2), (16, 5), (20, 2), (32, 3), (64, 4),
+         (100, 4), (255, 8),
          (1000, 3), (4096, 8)]
 
 
@@ -141,7 +145,7 @@ def test_div7_bits(n_bits):
     data = streams.random_bits(max(n_bits, 1), seed=n_bits)
     exp = seq.run(d, data, n_bits)
     for k in (1, 3, 7):
-        for var in ("P8", "B", "G", "R16"):
+        for var in ("P8", "B", "G"):
             got, st = gpu_run(d, data, n_bits, k=k, variant=VARIANTS[var], chunk_bytes=64)
             assert got == exp, (n_bits, k, var)
             if k == 7:
@@ -166,11 +170,11 @@ def test_r16_lane_replicated_bytes(n, m, offset):
 
 
 @pytest.mark.parametrize("kind", ["huffman13", "huffman17", "rand12", "rand16"])
-def test_r16_bit_mode_converging(kind):
-    """R16 in bit mode with chains that converge: the pending (one-step-late) count of a slot is
-    its own path's F-visits over the last widened byte, so the convergence collapse must settle it
-    per slot first.  Huffman decoders with 13 / 17 symbols (12 / 16 states,
-    self-synchronising codes) and near-permutation random bit DFAs, k >= 2, several chunkings."""
+def test_bit_mode_9_to_16_states_converging(kind):
+    """Bit-mode DFAs with 9-16 states and chains that converge (Huffman decoders with 13 / 17
+    symbols, near-permutation random bit DFAs), k >= 2, several chunkings.  A widened byte's count
+    (F-visits over 8 bits) depends on the source state, so the region-counting R16 is byte-mode only:
+    the library refuses it here and the auto choice (B) must be exact."""
     if kind.startswith("huffman"):
         ns = int(kind[7:])
         w = dfas.zipf_weights(ns, seed=ns)
@@ -184,12 +188,53 @@ def test_r16_bit_mode_converging(kind):
         n_bits = 2_000_003
         data = streams.random_bits(n_bits, seed=n)
     assert 9 <= d.n_states <= 16
+    with FSM.from_dfa(d) as f, pytest.raises(fsmspec.FsmError):
+        f.set_options(variant=VARIANTS["R16"])
     exp = seq.run(d, data, n_bits)
     for k in (2, 3, 4, 8):
         for chunk in (64, 256, 4096):
-            got, st = gpu_run(d, data, n_bits, k=k, variant=VARIANTS["R16"], chunk_bytes=chunk)
+            got, st = gpu_run(d, data, n_bits, k=k, chunk_bytes=chunk)
             assert got == exp, (kind, k, chunk, st)
-            assert st["variant"] == VARIANTS["R16"]
+            assert st["variant"] == VARIANTS["B"]
+
+
+def _accept_dfa(n, m, n_acc, alphabet, seed, ncls=None):
+    """A random (n, m) DFA with exactly n_acc accepting states (region-counting edge cases); with
+    ncls, its columns are those of a random ncls-symbol DFA under a random byte -> class map."""
+    rng = np.random.default_rng(seed)
+    if ncls:
+        r = dfas.random_dfa(n, m, seed=seed, alphabet=ncls)
+        table = np.ascontiguousarray(r.table[:, rng.integers(0, ncls, alphabet)])
+    else:
+        table = dfas.random_dfa(n, m, seed=seed, alphabet=alphabet).table
+    acc = np.zeros(n, np.uint8)
+    acc[rng.permutation(n)[:n_acc]] = 1
+    return dfas.DFA(table, int(seed % n), acc, False, f"acc_{n}_{n_acc}")
+
+
+@pytest.mark.parametrize("n,n_acc,alphabet", [(16, 0, 256), (16, 16, 256), (16, 8, 256), (16, 11, 256),
+                                               (15, 7, 256), (15, 8, 200), (12, 1, 256), (13, 12, 97),
+                                               (38, 5, 256), (38, 33, 256), (30, 15, 120)])
+def test_region_counting_partitions(n, n_acc, alphabet):
+    """R16 and CL count accepts by the destination id's region (accept-partitioned renumbering,
+    host_tables.h renumber_by_accept): F empty, F = Q, balanced partitions, the complement
+    orientation (|F| > |Q minus F|), a sink (alphabet < 256) and user start states that move.  Every k,
+    chunk sizes with ragged tails, unaligned starts; results in user ids against the oracle."""
+    d = _accept_dfa(n, 3, n_acc, alphabet, seed=8000 + 97 * n + n_acc + alphabet, ncls=None if n <= 16 else 20)
+    if alphabet < 256:
+        rng = np.random.default_rng(n)
+        data = rng.integers(0, alphabet, 500_003).astype(np.uint8)
+    else:
+        data = streams.splitmix_bytes(8100 + n + n_acc, 0, 500_003)
+    exp = seq.run(d, data)
+    for var in ("R16", "RG", "CL"):
+        if not fits(d, var):
+            continue
+        for k in (1, 2, 3, 4):
+            for chunk, offset in ((0, 0), (96, 0), (1024, 7)):
+                got, st = gpu_run(d, data, k=k, variant=VARIANTS[var], chunk_bytes=chunk, offset=offset)
+                assert got == exp, (var, k, chunk, offset, st)
+                assert st["variant"] == VARIANTS[var]
 
 
 def test_div7_closed_form_on_gpu():
@@ -538,7 +583,7 @@ def test_html_cl_large_k(k):
 
 
 # --------------------------------------------------------------------- production geometry
-FULL_CASES = [("P4", 4, 2), ("N8", 8, 2), ("P8", 8, 3), ("R16", 16, 2), ("B", 64, 4), ("G", 1000, 3),
+FULL_CASES = [("P4", 4, 2), ("N8", 8, 2), ("P8", 8, 3), ("R16", 16, 2), ("B", 64, 4), ("RG", 64, 4), ("RG", 200, 3), ("G", 1000, 3),
               ("HS", 3000, 3), ("CL", 0, 0)]
 
 

@@ -22,7 +22,7 @@ from paper_conf_ppopp_xiaja20_b200.fsmspec import FSM  # noqa: E402
 
 ST = {"a": 0, "b": 1, "c": 2, "d": 3}
 NAME = {v: k for k, v in ST.items()}
-VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8}
+VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8, "RG": 9}
 
 
 def dev(data: np.ndarray):
@@ -214,7 +214,7 @@ def test_hash_check_matches_nested(n, m, k):
     data = streams.splitmix_bytes(600 + n, 0, (3 << 20) + 11)
     exp = seq.run(d, data)
     for var in ("B", "G", "R16", "CL", "HS"):
-        if var == "R16" and n > 16:
+        if var == "R16" and n > 16:  # (byte mode here)
             continue
         with FSM.from_dfa(d) as f:
             buf, ptr = dev(data)

@@ -19,7 +19,7 @@ from oracle import seq  # noqa: E402
 from paper_conf_ppopp_xiaja20_b200 import fsmspec  # noqa: E402
 from paper_conf_ppopp_xiaja20_b200.fsmspec import FSM, run_multi  # noqa: E402
 
-V = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8}
+V = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8, "RG": 9}
 L = int(os.environ.get("SAN_BYTES", 1 << 20))
 
 

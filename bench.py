@@ -225,7 +225,7 @@ def cpu_model():
 def config_json(args, w):
     return {"workload": w["name"], "input_bytes": w["total"], "k": w["k"], "lookback_len": w.get("lookback"),
             "input_offset": args.offset,
-            "eager_window": w.get("eager", 0),
+            "eager_window": w.get("eager", 0), "lookback_width": w.get("width", 0),
             "n_states": int(w["dfa"].n_states), "parallelism": f"shard{args.gpus}",
             "l2": "input >> L2 (126 MB), no flush needed" if w["total"] > 4 * 126e6 else "L2 flushed between steps"}
 
@@ -288,6 +288,8 @@ def main():
     ap.add_argument("--lookback", type=int, default=-1,
                     help="look-back window bytes (R7; -1 = the config's default: c5 0, c1/c4 64, c2/c3 32)")
     ap.add_argument("--chunk", type=int, default=0)
+    ap.add_argument("--lb-width", type=int, default=0,
+                    help="look-back window walk over the top 4/8/12/16 image states only (0 = the whole image)")
     ap.add_argument("--eager", type=int, default=0,
                     help="eager-completion window bytes (NEXT-3): 0 = library default (128), 1 = off, 32..128")
     ap.add_argument("--tune", action="store_true",
@@ -351,13 +353,15 @@ def main():
     lookback = w["lookback"]
     eager = args.eager
     w["eager"] = eager
-    f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback, eager_window=eager)
+    f.set_options(variant=args.variant, chunk_bytes=args.chunk, lookback_len=lookback, eager_window=eager,
+                  lookback_width=args.lb_width)
+    w["width"] = args.lb_width
     tuning = None
     if args.tune:
         # offline, like fsm_create (not timed): the measured cost model picks the windows (and k)
         tuning = f.autotune(buf.data_ptr(), nsym, k_min=0 if args.tune_k else k, k_max=0 if args.tune_k else k)
         k, lookback, eager = tuning["k"], tuning["lookback_len"], tuning["eager_window"]
-        w["k"], w["lookback"], w["eager"] = k, lookback, eager
+        w["k"], w["lookback"], w["eager"], w["width"] = k, lookback, eager, tuning["lookback_width"]
         w["name"] = re.sub(r"spec-\d+", f"spec-{k} (tuned)", w["name"])
     res = torch.zeros(4, dtype=torch.int32, device=dev)
     small = total < 4 * 126_000_000

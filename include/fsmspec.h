@@ -169,6 +169,10 @@ typedef struct {
                                    (O(k), per-thread shared-memory buckets); the hash form is
                                    built for k > 8 (instantiated K = 12, 16) and falls back to Alg. 1
                                    where its scratch does not fit next to the table.  Identical results. */
+    uint32_t lookback_width;    /* look-back window walk (lookback_len >= 32): only the top lookback_width
+                                   states of the image (by preimage count, A5) are run through the window
+                                   and ranked; 0 = default (the whole image, up to FSM_KMAX), else 4, 8,
+                                   12 or 16.  Only the speculation (and so the re-execution work) changes. */
 } fsm_options;
 
 #define FSM_EAGER_OFF 1u
@@ -198,6 +202,7 @@ typedef struct {
     uint64_t max_miss_chain;    /* longest run of consecutive re-executed chunks on the true path */
     uint32_t chunk_bytes, threads_per_tile, variant, k_slots, lookback_len, preresolve;
     uint32_t check;             /* FSM_CHECK_NESTED or FSM_CHECK_HASH: the check the run used */
+    uint32_t lookback_width;    /* image states the look-back window walk ran (0: no window walk) */
 } fsm_stats;
 
 /* Synchronises the handle's stream (the counters live on the device). */
@@ -285,6 +290,7 @@ typedef struct {
     double hit_rate;            /* 1 - re-executed chunks / chunks, chosen configuration */
     int32_t variant;            /* chosen table variant (FSM_VARIANT_*), applied to the options */
     uint32_t preresolve;        /* chosen fsm_options.preresolve (0 = the default policy), applied */
+    uint32_t lookback_width;    /* chosen fsm_options.lookback_width (0 = the whole image), applied */
 } fsm_tuning;
 
 int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k_min, uint32_t k_max,

@@ -512,6 +512,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     if (o->eager_window > FSM_EAGER_OFF && (o->eager_window % 32 || o->eager_window > kExtWindow)) return FSM_EINVAL;
     if (o->preresolve > FSM_KMAX && o->preresolve != FSM_PRERESOLVE_NONE) return FSM_EINVAL;
     if (o->check > FSM_CHECK_HASH) return FSM_EINVAL;
+    if (o->lookback_width % 4 || o->lookback_width > FSM_KMAX) return FSM_EINVAL;
     f->opt.chunk_bytes = o->chunk_bytes;            // 0 = adaptive
     f->opt.threads_per_tile = o->threads_per_tile;  // 0 = auto
     f->opt.variant = o->variant;
@@ -519,6 +520,7 @@ extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
     f->opt.ctas_per_sm = o->ctas_per_sm;
     f->opt.grid_sms = o->grid_sms;
     f->opt.check = o->check;
+    f->opt.lookback_width = o->lookback_width;
     f->opt.lookback_len = o->lookback_len;
     f->opt.eager_window = o->eager_window;
     f->opt.preresolve = o->preresolve;
@@ -720,6 +722,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     p.ntiles = ntiles;
     p.k = r.k;
     p.lookback = f->opt.lookback_len > 1 ? f->opt.lookback_len : 0;
+    p.lb_width = f->opt.lookback_width ? f->opt.lookback_width : KMAX;
     p.eager_window = f->opt.eager_window == 0 ? kExtWindow : f->opt.eager_window == FSM_EAGER_OFF ? 0u : f->opt.eager_window;
     p.preresolve = preresolve_of(f);
     if (dbg && f->dbg_n) {
@@ -817,6 +820,7 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
     f->last.variant = var;
     f->last.k_slots = K;
     f->last.lookback_len = p.lookback;
+    f->last.lookback_width = p.lookback >= 32 ? p.lb_width : 0;
     f->last.preresolve = p.preresolve;
     f->last_head = head;
     f->last.check = hash ? FSM_CHECK_HASH : FSM_CHECK_NESTED;
@@ -1252,6 +1256,7 @@ struct TuneCand {
     uint32_t k, lookback, eager;
     int32_t variant = FSM_VARIANT_AUTO;
     uint32_t preresolve = 0;
+    uint32_t width = 0;
     double ms = 0, hit = 0;
 };
 }  // namespace
@@ -1264,6 +1269,7 @@ static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom
     o.eager_window = c.eager;
     o.variant = c.variant;
     o.preresolve = c.preresolve;
+    o.lookback_width = c.width;
     o.merge = FSM_MERGE_PARALLEL;
     int rc = fsm_set_options(f, &o);
     if (rc) return rc;
@@ -1307,11 +1313,12 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
     CK(cudaEventCreate(&e1));
     std::vector<TuneCand> tried;
     int rc = FSM_OK;
-    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg, int32_t var = -2, uint32_t pre = 0) -> int {
+    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg, int32_t var = -2, uint32_t pre = 0, uint32_t w = 0) -> int {
         if (var == -2) var = saved.variant;  // stages 1-2: the handle's own variant choice
         for (const TuneCand &c : tried)
-            if (c.k == k && c.lookback == lb && c.eager == eg && c.variant == var && c.preresolve == pre) return FSM_OK;
-        TuneCand c{k, lb, eg, var, pre};
+            if (c.k == k && c.lookback == lb && c.eager == eg && c.variant == var && c.preresolve == pre && c.width == w)
+                return FSM_OK;
+        TuneCand c{k, lb, eg, var, pre, w};
         int r = time_candidate(f, input, n, len / sym_per_byte, c, e0, e1);
         if (r == FSM_OK) tried.push_back(c);
         return r;
@@ -1339,6 +1346,17 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
                 for (uint32_t eg : {FSM_EAGER_OFF, 0u})
                     if (rc == FSM_OK) rc = run(k, lb, eg);
     }
+    // stage 2b: the window walk over the top 4 / 8 image states only (R7 width) at the best windowed setting
+    if (rc == FSM_OK) {
+        const TuneCand *b = nullptr;
+        for (const TuneCand &c : tried)
+            if (c.lookback >= 32 && (!b || c.ms < b->ms)) b = &c;
+        if (b) {
+            const TuneCand bw = *b;
+            for (uint32_t w : {4u, 8u})
+                if (rc == FSM_OK) rc = run(bw.k, bw.lookback, bw.eager, bw.variant, 0, w);
+        }
+    }
     if (rc == FSM_OK) rc = run(1, 0, FSM_EAGER_OFF);  // the paper's plain spec-1, for reference
     // stage 3: every table variant the DFA fits, at the best (k, window, eager) so far
     if (rc == FSM_OK) {
@@ -1348,7 +1366,8 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
         const TuneCand best_so_far = *b;
         const int base = saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;  // what stages 1-2 ran
         for (int v = 0; v < 10 && rc == FSM_OK; v++)
-            if (f->d_img[v] && v != base) rc = run(best_so_far.k, best_so_far.lookback, best_so_far.eager, v);
+            if (f->d_img[v] && v != base)
+                rc = run(best_so_far.k, best_so_far.lookback, best_so_far.eager, v, 0, best_so_far.width);
     }
     // stage 4: R5 pre-resolution (top-1 vs every candidate) at the best setting so far
     if (rc == FSM_OK) {
@@ -1358,7 +1377,7 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
         const TuneCand bb = *b;
         if (bb.k > 1)
             for (uint32_t pre : {1u, (uint32_t)FSM_KMAX})
-                if (rc == FSM_OK) rc = run(bb.k, bb.lookback, bb.eager, bb.variant, pre);
+                if (rc == FSM_OK) rc = run(bb.k, bb.lookback, bb.eager, bb.variant, pre, bb.width);
     }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
@@ -1382,6 +1401,8 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
     out->variant = best->variant != FSM_VARIANT_AUTO ? best->variant
                  : saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;
     out->preresolve = best->preresolve;
+    out->lookback_width = best->width;
+    f->opt.lookback_width = best->width;
     f->opt.lookback_len = best->lookback;
     f->opt.eager_window = out->eager_window;
     f->opt.variant = out->variant;

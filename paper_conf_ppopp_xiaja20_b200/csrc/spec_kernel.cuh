@@ -1,6 +1,7 @@
 // spec_kernel.cuh -- a3 look-back speculation with a window (reading R7), as a pre-pass.
 //
-// For every chunk (start byte b): the image of x[b-Lw-1] (the host look-back table) is run
+// For every chunk (start byte b): the image of x[b-Lw-1] (the host look-back table; its top
+// lb_width states by preimage count when the option narrows the walk) is run
 // through the Lw bytes x[b-Lw .. b) and the reached states are ranked by multiplicity (how many
 // image states reach each), ties to the smaller (user) id; the top k + kExt distinct states are written
 // to spec[chunk][0 .. k + kExt) (0xFFFF = none).  Chunks whose window would reach before the start
@@ -35,7 +36,7 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
             out[written++] = (uint16_t)start_state;
         } else if (b >= Lw + 1 + p.head && p.aligned) {
             const uint32_t c0 = __ldg(p.in + b - Lw - 1);
-            const uint32_t ni = __ldg(p.nimg + c0);
+            const uint32_t ni = min((uint32_t)__ldg(p.nimg + c0), p.lb_width);  // the top lb_width (A5 rank)
             // the image chains run in the table variant's own hot-loop form (its step(), on groups of
             // 4 chains, only as many groups as the image has states); ids are recovered at the end
             uint32_t cur[KMAX / 4][4], acc[KMAX / 4][4], accf[KMAX / 4][4];

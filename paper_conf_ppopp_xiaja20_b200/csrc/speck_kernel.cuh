@@ -44,7 +44,12 @@ constexpr uint32_t kLockstepWindow = 256;  // Alg. 2 buckets per thread (reading
 // caps them for large K.
 // (K = 2, 3 at 768 threads get 85 registers: the multi-chain prologue spills at 64; measured
 // +6 % over 1024 threads for (8, 2, k=2).)
-__host__ __device__ constexpr int max_threads(int K, int = -1) { return K == 1 ? 1024 : K <= 3 ? 768 : K <= 6 ? 512 : 256; }
+// R16 / RG at K = 4 (their chains converge within a few bytes, after which one LDS-latency-bound
+// chain per thread remains): 768 threads (85 registers) instead of 512 (128).
+__host__ __device__ constexpr int max_threads(int K, int var = -1)
+{
+    return K == 1 ? 1024 : K <= 3 ? 768 : (K == 4 && (var == 8 || var == 9)) ? 768 : K <= 6 ? 512 : 256;
+}
 __host__ __device__ constexpr int min_blocks(int) { return 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
 

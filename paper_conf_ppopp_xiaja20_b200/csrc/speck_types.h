@@ -118,6 +118,7 @@ struct Params {
     // (count = steps - that).
     uint32_t rc_t, rc_comp;
     uint32_t r_logl;               // RG variant: log2 of the lanes that share one table copy
+    uint32_t lb_width;             // window look-back: image states run through the window (4..16)
 };
 
 }  // namespace speck

@@ -37,14 +37,14 @@ class fsm_options(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
                 ("variant", ctypes.c_int32), ("merge", ctypes.c_uint32), ("ctas_per_sm", ctypes.c_uint32),
                 ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32), ("preresolve", ctypes.c_uint32),
-                ("grid_sms", ctypes.c_uint32), ("check", ctypes.c_uint32)]
+                ("grid_sms", ctypes.c_uint32), ("check", ctypes.c_uint32), ("lookback_width", ctypes.c_uint32)]
 
 
 class fsm_tuning(ctypes.Structure):
     _fields_ = [("k", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32),
                 ("candidates", ctypes.c_uint32), ("sample_len", ctypes.c_uint64), ("best_gbs", ctypes.c_double),
                 ("paper_gbs", ctypes.c_double), ("hit_rate", ctypes.c_double), ("variant", ctypes.c_int32),
-                ("preresolve", ctypes.c_uint32)]
+                ("preresolve", ctypes.c_uint32), ("lookback_width", ctypes.c_uint32)]
 
 
 class fsm_stats(ctypes.Structure):
@@ -55,7 +55,7 @@ class fsm_stats(ctypes.Structure):
                 ("eager_resolved", ctypes.c_uint64), ("max_miss_chain", ctypes.c_uint64),
                 ("chunk_bytes", ctypes.c_uint32), ("threads_per_tile", ctypes.c_uint32),
                 ("variant", ctypes.c_uint32), ("k_slots", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32),
-                ("preresolve", ctypes.c_uint32), ("check", ctypes.c_uint32)]
+                ("preresolve", ctypes.c_uint32), ("check", ctypes.c_uint32), ("lookback_width", ctypes.c_uint32)]
 
 
 class fsm_shard_map(ctypes.Structure):
@@ -241,9 +241,10 @@ class FSM:
 
     def set_options(self, chunk_bytes: int = 0, threads_per_tile: int = 0, variant: int = FSM_VARIANT_AUTO,
                     merge: int = FSM_MERGE_PARALLEL, ctas_per_sm: int = 0, lookback_len: int = 0,
-                    eager_window: int = 0, preresolve: int = 0, grid_sms: int = 0, check: int = 0) -> None:
+                    eager_window: int = 0, preresolve: int = 0, grid_sms: int = 0, check: int = 0,
+                    lookback_width: int = 0) -> None:
         o = fsm_options(chunk_bytes, threads_per_tile, variant, merge, ctas_per_sm, lookback_len, eager_window,
-                        preresolve, grid_sms, check)
+                        preresolve, grid_sms, check, lookback_width)
         _check(lib().fsm_set_options(self._h, ctypes.byref(o)), "fsm_set_options")
 
     def options(self) -> dict:

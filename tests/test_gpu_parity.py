@@ -440,6 +440,22 @@ def test_lookback_window_parity(lookback):
                 assert st["lookback_len"] == lookback
 
 
+@pytest.mark.parametrize("width", [4, 8, 12])
+def test_lookback_width_parity(width):
+    """The window walk over the top 4 / 8 / 12 image states only (fsm_options.lookback_width): exact
+    results, the width reported; widths that are not multiples of 4 (or > 16) are rejected."""
+    for name, d, data, length in _wl_cases():
+        exp = seq.run(d, data, length)
+        for k in (1, 3):
+            got, st = gpu_run(d, data, length, k=k, chunk_bytes=512, lookback_len=64, lookback_width=width)
+            assert got == exp, (name, width, k, st)
+            assert st["lookback_width"] == width and st["lookback_len"] == 64
+    with FSM.from_dfa(dfas.html_tokenizer()) as f:
+        for bad in (2, 5, 20):
+            with pytest.raises(fsmspec.FsmError):
+                f.set_options(lookback_len=64, lookback_width=bad)
+
+
 def test_lookback_window_reduces_misses():
     d = dfas.html_tokenizer()
     data = streams.html_bytes(4_000_000, 5)

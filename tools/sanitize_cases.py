@@ -42,6 +42,8 @@ def main():
         ("P8", dfas.random_dfa(8, 3, seed=3), (1, 3)),
         ("R16", dfas.random_dfa(16, 3, seed=4), (1, 2)),
         ("B", dfas.random_dfa(64, 4, seed=5), (1, 4)),
+        ("RG", dfas.random_dfa(64, 4, seed=5), (1, 4)),
+        ("RG", dfas.random_dfa(200, 3, seed=8), (1, 2)),
         ("CL", dfas.html_tokenizer(), (1, 2)),
         ("G", dfas.random_dfa(1000, 3, seed=6), (1, 2)),
         ("HS", dfas.random_dfa(3000, 3, seed=7), (1,)),

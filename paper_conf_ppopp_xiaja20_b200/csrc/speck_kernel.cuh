@@ -44,11 +44,11 @@ constexpr uint32_t kLockstepWindow = 256;  // Alg. 2 buckets per thread (reading
 // caps them for large K.
 // (K = 2, 3 at 768 threads get 85 registers: the multi-chain prologue spills at 64; measured
 // +6 % over 1024 threads for (8, 2, k=2).)
-// R16 / RG at K = 4 (their chains converge within a few bytes, after which one LDS-latency-bound
-// chain per thread remains): 768 threads (85 registers) instead of 512 (128).
+// B / R16 / RG at K = 4 (their chains converge within a few bytes, after which one LDS-bound chain
+// per thread remains): 768 threads (80 registers) instead of 512 (128).
 __host__ __device__ constexpr int max_threads(int K, int var = -1)
 {
-    return K == 1 ? 1024 : K <= 3 ? 768 : (K == 4 && (var == 8 || var == 9)) ? 768 : K <= 6 ? 512 : 256;
+    return K == 1 ? 1024 : K <= 3 ? 768 : (K == 4 && (var == 2 || var == 8 || var == 9)) ? 768 : K <= 6 ? 512 : 256;
 }
 __host__ __device__ constexpr int min_blocks(int) { return 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows
@@ -590,8 +590,9 @@ struct TableRep {
     {
         return comp ? (uint32_t)n - (acc + accf) : acc + accf;
     }
-    // symbol part of the address of byte j of w.  The chain and the count are on the FMA pipe, so
-    // R16's odd bytes combine the two halves with a shift-add (LEA, ALU pipe) instead of an IMAD.
+    // symbol part of the address of byte j of w.  R16's odd bytes combine the two halves with a
+    // shift-add (LEA, ALU pipe) instead of an IMAD: measured 0-2 % faster than IMADs on every byte,
+    // although ncu shows the ALU pipe 82 % busy and the FMA pipe 20 %.
     __device__ __forceinline__ uint32_t sym(uint32_t w, int j) const
     {
         const uint32_t m = GROUPED ? mlo : 0x03030303u;

@@ -84,7 +84,7 @@ def test_fig1_worked_example(var, k):
 
 # --------------------------------------------------------------------- C1-shaped text
 @pytest.mark.parametrize("var", ["P4", "P8", "N8", "R16", "B", "G", "HS", "CL"])
-@pytest.mark.parametrize("chunk", [0, 64, 96, 4096])
+@pytest.mark.parametrize("chunk", [0, 64, 96, 4096, 8192])
 def test_c_comment_text(var, chunk):
     d = dfas.c_comment(True)
     data = streams.c_source(300_001, seed=streams.MASTER_SEED + 1, comment_frac=0.3)
@@ -110,7 +110,7 @@ def test_random_dfa_parity(n, m):
         if not fits(d, var):
             continue
         for k in sorted({1, 2, 3, min(m, 16), min(n, 16), 5, 16} & set(range(1, min(n, 16) + 1))):
-            for chunk in (64, 1024):
+            for chunk in (64, 1024, 8192):
                 got, st = gpu_run(d, data, k=k, variant=VARIANTS[var], chunk_bytes=chunk)
                 assert got == exp, (n, m, var, k, chunk, st)
                 if k >= m:
@@ -126,6 +126,20 @@ def test_lengths_and_alignment(length, offset):
     for k in (1, 2, 3):
         got, _ = gpu_run(d, data, length, k=k, offset=offset, chunk_bytes=64)
         assert got == exp, (length, offset, k)
+
+
+@pytest.mark.parametrize("length", [1 << 20, (64 << 20) + 5, 300 << 20])
+def test_default_geometry_power_of_two_chunks(length):
+    """pick_geometry's wave model: default chunks are powers of two up to 8 KiB (4 KiB for G),
+    results exact at every size."""
+    d = dfas.random_dfa(16, 2, seed=77)
+    data = streams.splitmix_bytes(78, 0, length)
+    exp = seq.run(d, data)
+    for var, k, cap in (("R16", 2, 8192), ("G", 1, 4096)):
+        got, st = gpu_run(d, data, k=k, variant=VARIANTS[var])
+        assert got == exp, (var, length, st)
+        c = st["chunk_bytes"]
+        assert 64 <= c <= cap and c & (c - 1) == 0, st
 
 
 def test_out_of_alphabet_is_reported():

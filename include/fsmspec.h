@@ -136,7 +136,8 @@ int fsm_run_spec_k_host(fsm_t *f, const uint8_t *host_input, uint64_t len, uint3
 
 /* Tuning knobs; zero fields keep the current value.  Applied to subsequent runs. */
 typedef struct {
-    uint32_t chunk_bytes;       /* bytes per chunk (per thread), multiple of 32; 0 = adaptive */
+    uint32_t chunk_bytes;       /* bytes per chunk (per thread), multiple of 32, <= 16384 (8192 in bit
+                                   mode); 0 = adaptive (power-of-two chunks by a wave model) */
     uint32_t threads_per_tile;  /* chunks per tile (CTA size), 64 .. 1024, multiple of 32 */
     int32_t variant;            /* FSM_VARIANT_*; FSM_VARIANT_AUTO = by state count */
     uint32_t merge;             /* FSM_MERGE_* */

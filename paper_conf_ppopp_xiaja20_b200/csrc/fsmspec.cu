@@ -501,8 +501,10 @@ extern "C" int fsm_set_stream(fsm_t *f, void *s)
 extern "C" int fsm_set_options(fsm_t *f, const fsm_options *o)
 {
     if (!f || !o) return FSM_EINVAL;
-    // chunk <= 8 KiB keeps 32-tile look-back windows of counts inside 32 bits (8 per byte in bit mode)
-    if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > 8192)) return FSM_EINVAL;
+    // chunk <= 8 KiB (16 KiB in byte mode) keeps 32-tile look-back windows of counts inside 32 bits
+    // (up to 8 accepts per byte in bit mode, 1 in byte mode)
+    const uint32_t max_chunk = f->mode == FSM_INPUT_BITS_MSB ? 8192u : 16384u;
+    if (o->chunk_bytes && (o->chunk_bytes % 32 || o->chunk_bytes > max_chunk)) return FSM_EINVAL;
     if (o->threads_per_tile && (o->threads_per_tile % 32 || o->threads_per_tile < 32 || o->threads_per_tile > 1024))
         return FSM_EINVAL;
     if (o->variant < FSM_VARIANT_AUTO || o->variant > FSM_VARIANT_RG) return FSM_EINVAL;
@@ -602,8 +604,8 @@ static int variant_of(const fsm *f, int force, uint32_t k = 1)
 }
 
 // Geometry: T chunks per tile (CTA threads), chunk bytes.  Large inputs: the largest CTA the
-// register budget allows for K and 8 KiB chunks (4 KiB for G / HS).  Small inputs: shrink the CTA,
-// then the chunk, so that every SM still gets a tile.
+// register budget allows for K and 16 KiB chunks (8 KiB in bit mode, 4 KiB for G / HS).  Small
+// inputs: shrink the CTA, then the chunk, so that every SM still gets a tile.
 static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, int var, uint32_t &T, uint32_t &chunk)
 {
     const uint32_t tmax = (uint32_t)max_threads(K, var);
@@ -614,13 +616,15 @@ static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, int var, uint
         chunk = f->opt.chunk_bytes;
         return;
     }
-    // Power-of-two chunks up to 8 KiB (4 KiB for the L2-table variants G / HS), chosen by a wave
+    // Power-of-two chunks up to 16 KiB in byte mode, 8 KiB in bit mode (the counts' 32-bit range, see
+    // fsm_set_options) and 4 KiB for the L2-table variants G / HS, chosen by a wave
     // model: a persistent grid of one CTA per SM takes tiles dynamically, so a run costs about
     // ceil(tiles / SMs) x (chunk + a per-chunk overhead of ~1 KiB-equivalents: speculation, the window
     // walk, the merge).  Measured on 8 GiB against 4 KiB: C4 k = 1 2590 -> 2992, (64, 4, k = 4)
     // 2349 -> 2534, (16, 2, k = 2) 3467 -> 3578 GB/s; C3 (G) 1191 at 4 KiB vs 1058 at 8 KiB.
-    // Chunks that are not powers of two measured 2-25 % slower (7328 B: C4 2225 GB/s).
-    const uint64_t cap = (var == VAR_G || var == VAR_HS) ? 4096 : 8192;
+    // Chunks that are not powers of two measured 2-25 % slower (7328 B: C4 2225 GB/s).  16 KiB
+    // against 8 KiB on 8 GiB: C4 2987 -> 3190, (64, 4, k = 4) 2535 -> 2634, (8, 2, k = 2) 4391 -> 4481.
+    const uint64_t cap = (var == VAR_G || var == VAR_HS) ? 4096 : f->mode == FSM_INPUT_BITS_MSB ? 8192 : 16384;
     const uint64_t te = split_kernel(var, K) && T >= 64 ? T - 32 : T;  // chunks per tile
     uint64_t best = 0, best_cost = ~0ull;
     for (uint64_t c = cap; c >= 64; c >>= 1) {

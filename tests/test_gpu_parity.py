@@ -38,6 +38,10 @@ def gpu_run(dfa, data, length=None, k=1, offset=0, **opt):
 VARIANTS = {"P4": 0, "P8": 1, "B": 2, "G": 3, "HS": 5, "CL": 6, "N8": 7, "R16": 8, "RG": 9}
 
 
+def dfa_bits(dfa):
+    return bool(dfa.bit_mode)
+
+
 def fits(dfa, var):
     n = dfa.n_states + (1 if (not dfa.bit_mode and dfa.alphabet < 256) else 0)
     # R16 and CL use region counting (accept-partitioned ids): byte mode only
@@ -84,7 +88,7 @@ def test_fig1_worked_example(var, k):
 
 # --------------------------------------------------------------------- C1-shaped text
 @pytest.mark.parametrize("var", ["P4", "P8", "N8", "R16", "B", "G", "HS", "CL"])
-@pytest.mark.parametrize("chunk", [0, 64, 96, 4096, 8192])
+@pytest.mark.parametrize("chunk", [0, 64, 96, 4096, 16384])
 def test_c_comment_text(var, chunk):
     d = dfas.c_comment(True)
     data = streams.c_source(300_001, seed=streams.MASTER_SEED + 1, comment_frac=0.3)
@@ -110,7 +114,7 @@ def test_random_dfa_parity(n, m):
         if not fits(d, var):
             continue
         for k in sorted({1, 2, 3, min(m, 16), min(n, 16), 5, 16} & set(range(1, min(n, 16) + 1))):
-            for chunk in (64, 1024, 8192):
+            for chunk in (64, 1024, 8192 if dfa_bits(d) else 16384):
                 got, st = gpu_run(d, data, k=k, variant=VARIANTS[var], chunk_bytes=chunk)
                 assert got == exp, (n, m, var, k, chunk, st)
                 if k >= m:
@@ -130,16 +134,29 @@ def test_lengths_and_alignment(length, offset):
 
 @pytest.mark.parametrize("length", [1 << 20, (64 << 20) + 5, 300 << 20])
 def test_default_geometry_power_of_two_chunks(length):
-    """pick_geometry's wave model: default chunks are powers of two up to 8 KiB (4 KiB for G),
+    """pick_geometry's wave model: default chunks are powers of two up to 16 KiB (4 KiB for G),
     results exact at every size."""
     d = dfas.random_dfa(16, 2, seed=77)
     data = streams.splitmix_bytes(78, 0, length)
     exp = seq.run(d, data)
-    for var, k, cap in (("R16", 2, 8192), ("G", 1, 4096)):
+    for var, k, cap in (("R16", 2, 16384), ("G", 1, 4096)):
         got, st = gpu_run(d, data, k=k, variant=VARIANTS[var])
         assert got == exp, (var, length, st)
         c = st["chunk_bytes"]
         assert 64 <= c <= cap and c & (c - 1) == 0, st
+
+
+def test_chunk_limits():
+    """fsm_set_options: chunks up to 16 KiB in byte mode, 8 KiB in bit mode (32-bit tile-window counts)."""
+    with FSM.from_dfa(dfas.random_dfa(8, 2, seed=1)) as f:
+        f.set_options(chunk_bytes=16384)
+        for bad in (16416, 32768, 100):
+            with pytest.raises(fsmspec.FsmError):
+                f.set_options(chunk_bytes=bad)
+    with FSM.from_dfa(dfas.div7()) as f:
+        f.set_options(chunk_bytes=8192)
+        with pytest.raises(fsmspec.FsmError):
+            f.set_options(chunk_bytes=16384)
 
 
 def test_out_of_alphabet_is_reported():
@@ -620,7 +637,7 @@ FULL_CASES = [("P4", 4, 2), ("N8", 8, 2), ("P8", 8, 3), ("R16", 16, 2), ("B", 64
 @pytest.mark.parametrize("var,n,m", FULL_CASES)
 def test_full_geometry_parity(var, n, m):
     """Every table variant at the bench's launch geometry (inputs large enough that pick_geometry
-    chooses the maximal tile and chunks of several KiB -- up to 8 KiB, 4 KiB for the L2-table
+    chooses the maximal tile and chunks of several KiB -- up to 16 KiB, 4 KiB for the L2-table
     variants G / HS -- split kernels where the policy splits) against the
     oracle, k = 1 and 2, with the default look-back and eager completion."""
     L = 1280 << 20  # > 148 SMs x 1024 threads x 8 KiB: the maximal tile, two waves of tiles
@@ -637,6 +654,6 @@ def test_full_geometry_parity(var, n, m):
             f.set_options(variant=VARIANTS[var], lookback_len=64 if var == "CL" else 0)
             assert f.run_spec_k(ptr, L, k) == exp, (var, k)
             st = f.stats()
-            assert 2048 <= st["chunk_bytes"] <= (4096 if var in ("G", "HS") else 8192), st
+            assert 2048 <= st["chunk_bytes"] <= (4096 if var in ("G", "HS") else 16384), st
             assert st["threads_per_tile"] >= 224, st
             assert st["variant"] == VARIANTS[var]

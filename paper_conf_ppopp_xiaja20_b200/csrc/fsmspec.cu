@@ -611,7 +611,7 @@ static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, int var, uint
     const uint32_t tmax = (uint32_t)max_threads(K, var);
     T = f->opt.threads_per_tile ? std::min<uint32_t>(f->opt.threads_per_tile, tmax) : tmax;
     if (!f->opt.threads_per_tile)
-        while (T > 128 && len_bytes < (uint64_t)f->num_sms * T * 4096) T >>= 1;
+        while (T > 128 && len_bytes < (uint64_t)f->num_sms * T * 4096) T = std::max(128u, (T >> 1) & ~31u);
     if (f->opt.chunk_bytes) {
         chunk = f->opt.chunk_bytes;
         return;
@@ -719,7 +719,8 @@ static int prepare_run(fsm *f, const RunSpec &r, Prepared &out)
         const uint32_t tb = var == VAR_HS ? 0u : f->img_bytes[var];
         if (hash && !f->opt.threads_per_tile && f->opt.check == FSM_CHECK_HASH) {
             // Alg. 2 requested: halve the tile until its per-thread columns fit next to the table
-            while (T > 64 && Layout(T, K, scratch_offset(var, tb), false, true).total > kMaxSmem) T >>= 1;
+            while (T > 64 && Layout(T, K, scratch_offset(var, tb), false, true).total > kMaxSmem)
+                T = std::max(64u, (T >> 1) & ~31u);  // whole warps (max_threads need not be a power of two)
         }
         if (hash && Layout(T, K, scratch_offset(var, tb), false, true).total > kMaxSmem) hash = false;  // Alg. 1
         if (split)  // the double-buffered layout must fit next to the table (HS sizes its hot rows after)

@@ -45,10 +45,13 @@ constexpr uint32_t kLockstepWindow = 256;  // Alg. 2 buckets per thread (reading
 // (K = 2, 3 at 768 threads get 85 registers: the multi-chain prologue spills at 64; measured
 // +6 % over 1024 threads for (8, 2, k=2).)
 // B / R16 / RG at K = 4 (their chains converge within a few bytes, after which one LDS-bound chain
-// per thread remains): 768 threads (80 registers) instead of 512 (128).
+// per thread remains): 768 threads (80 registers) instead of 512 (128).  The shared-memory tables
+// at K = 8, 12: 384 / 320 threads (164 / 168 registers, no spills) instead of 256; K = 16 keeps 256
+// (at 288 threads ptxas caps it at 168 registers and spills 1.2 KB).
 __host__ __device__ constexpr int max_threads(int K, int var = -1)
 {
-    return K == 1 ? 1024 : K <= 3 ? 768 : (K == 4 && (var == 2 || var == 8 || var == 9)) ? 768 : K <= 6 ? 512 : 256;
+    return K == 1 ? 1024 : K <= 3 ? 768 : (K == 4 && (var == 2 || var == 8 || var == 9)) ? 768 : K <= 6 ? 512
+         : ((var == 2 || var == 6 || var == 8 || var == 9) && K <= 12) ? (K <= 8 ? 384 : 320) : 256;
 }
 __host__ __device__ constexpr int min_blocks(int) { return 1; }
 constexpr uint32_t kPackedTableBytes = 65536;  // 256 symbols x 256-byte lane-replicated rows

@@ -292,6 +292,8 @@ typedef struct {
     int32_t variant;            /* chosen table variant (FSM_VARIANT_*), applied to the options */
     uint32_t preresolve;        /* chosen fsm_options.preresolve (0 = the default policy), applied */
     uint32_t lookback_width;    /* chosen fsm_options.lookback_width (0 = the whole image), applied */
+    uint32_t chunk_bytes;       /* chosen fsm_options.chunk_bytes (0 = adaptive), applied; tuned only
+                                   when the handle's chunk_bytes was adaptive */
 } fsm_tuning;
 
 int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32_t k_min, uint32_t k_max,

@@ -619,8 +619,8 @@ static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, int var, uint
     // Power-of-two chunks up to 16 KiB in byte mode, 8 KiB in bit mode (the counts' 32-bit range, see
     // fsm_set_options) and 4 KiB for the L2-table variants G / HS, chosen by a wave
     // model: a persistent grid of one CTA per SM takes tiles dynamically, so a run costs about
-    // ceil(tiles / SMs) x (chunk + a per-chunk overhead of ~1 KiB-equivalents: speculation, the window
-    // walk, the merge).  Measured on 8 GiB against 4 KiB: C4 k = 1 2590 -> 2992, (64, 4, k = 4)
+    // ceil(tiles / SMs) x (chunk + a per-chunk overhead of ~K KiB-equivalents: speculation, the K-chain
+    // prologue, the window walk, the merge; C4 k = 4: 16 KiB 1832 vs 8 KiB 1439 GB/s).  Measured on 8 GiB against 4 KiB: C4 k = 1 2590 -> 2992, (64, 4, k = 4)
     // 2349 -> 2534, (16, 2, k = 2) 3467 -> 3578 GB/s; C3 (G) 1191 at 4 KiB vs 1058 at 8 KiB.
     // Chunks that are not powers of two measured 2-25 % slower (7328 B: C4 2225 GB/s).  16 KiB
     // against 8 KiB on 8 GiB: C4 2987 -> 3190, (64, 4, k = 4) 2535 -> 2634, (8, 2, k = 2) 4391 -> 4481.
@@ -629,7 +629,7 @@ static void pick_geometry(const fsm *f, uint64_t len_bytes, int K, int var, uint
     uint64_t best = 0, best_cost = ~0ull;
     for (uint64_t c = cap; c >= 64; c >>= 1) {
         const uint64_t tiles = std::max<uint64_t>(1, (len_bytes + te * c - 1) / (te * c));
-        const uint64_t cost = (tiles + f->num_sms - 1) / f->num_sms * (c + 1024);
+        const uint64_t cost = (tiles + f->num_sms - 1) / f->num_sms * (c + 1024ull * K);
         if (cost < best_cost) {
             best = c;
             best_cost = cost;
@@ -1276,6 +1276,8 @@ struct TuneCand {
     int32_t variant = FSM_VARIANT_AUTO;
     uint32_t preresolve = 0;
     uint32_t width = 0;
+    uint32_t chunk = 0;  // 0 = the geometry's choice
+    uint32_t used_chunk = 0;
     double ms = 0, hit = 0;
 };
 }  // namespace
@@ -1289,6 +1291,7 @@ static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom
     o.variant = c.variant;
     o.preresolve = c.preresolve;
     o.lookback_width = c.width;
+    o.chunk_bytes = c.chunk;
     o.merge = FSM_MERGE_PARALLEL;
     int rc = fsm_set_options(f, &o);
     if (rc) return rc;
@@ -1299,6 +1302,7 @@ static int time_candidate(fsm *f, const uint8_t *in, uint64_t len, uint64_t geom
     fsm_stats st;
     if ((rc = fsm_get_stats(f, &st))) return rc;
     c.hit = st.chunks ? 1.0 - (double)st.reexec_true / (double)st.chunks : 1.0;
+    c.used_chunk = st.chunk_bytes;
     float t[3];
     for (int i = 0; i < 3; i++) {
         CK(cudaEventRecord(e0, f->stream));
@@ -1332,12 +1336,15 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
     CK(cudaEventCreate(&e1));
     std::vector<TuneCand> tried;
     int rc = FSM_OK;
-    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg, int32_t var = -2, uint32_t pre = 0, uint32_t w = 0) -> int {
+    auto run = [&](uint32_t k, uint32_t lb, uint32_t eg, int32_t var = -2, uint32_t pre = 0, uint32_t w = 0,
+                   uint32_t ch = 0) -> int {
         if (var == -2) var = saved.variant;  // stages 1-2: the handle's own variant choice
+        if (ch == 0) ch = saved.chunk_bytes;
         for (const TuneCand &c : tried)
-            if (c.k == k && c.lookback == lb && c.eager == eg && c.variant == var && c.preresolve == pre && c.width == w)
+            if (c.k == k && c.lookback == lb && c.eager == eg && c.variant == var && c.preresolve == pre && c.width == w &&
+                c.chunk == ch)
                 return FSM_OK;
-        TuneCand c{k, lb, eg, var, pre, w};
+        TuneCand c{k, lb, eg, var, pre, w, ch};
         int r = time_candidate(f, input, n, len / sym_per_byte, c, e0, e1);
         if (r == FSM_OK) tried.push_back(c);
         return r;
@@ -1398,6 +1405,19 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
             for (uint32_t pre : {1u, (uint32_t)FSM_KMAX})
                 if (rc == FSM_OK) rc = run(bb.k, bb.lookback, bb.eager, bb.variant, pre, bb.width);
     }
+    // stage 5: chunk size (half and double the geometry's choice) at the best setting so far, when the
+    // caller left it adaptive and the sample is the whole input (a prefix has other tile waves: it
+    // measured 16 KiB chunks 15 % slow on a 2 GiB prefix of C4 that are 16 % fast on the 8 GiB run)
+    if (rc == FSM_OK && saved.chunk_bytes == 0 && n == len) {
+        const TuneCand *b = nullptr;
+        for (const TuneCand &c : tried)
+            if (c.k >= k_min && c.k <= k_max && (!b || c.ms < b->ms)) b = &c;
+        const TuneCand bb = *b;
+        const uint32_t cmax = bits ? 8192u : 16384u;
+        for (uint32_t ch : {bb.used_chunk / 2, bb.used_chunk * 2})
+            if (rc == FSM_OK && ch >= 64 && ch % 32 == 0 && ch <= cmax)
+                rc = run(bb.k, bb.lookback, bb.eager, bb.variant, bb.preresolve, bb.width, ch);
+    }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     f->opt = saved;
@@ -1421,7 +1441,9 @@ extern "C" int fsm_autotune(fsm_t *f, const uint8_t *input, uint64_t len, uint32
                  : saved.variant != FSM_VARIANT_AUTO ? saved.variant : f->auto_variant;
     out->preresolve = best->preresolve;
     out->lookback_width = best->width;
+    out->chunk_bytes = best->chunk;
     f->opt.lookback_width = best->width;
+    f->opt.chunk_bytes = best->chunk;
     f->opt.lookback_len = best->lookback;
     f->opt.eager_window = out->eager_window;
     f->opt.variant = out->variant;

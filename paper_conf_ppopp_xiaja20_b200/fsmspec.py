@@ -44,7 +44,7 @@ class fsm_tuning(ctypes.Structure):
     _fields_ = [("k", ctypes.c_uint32), ("lookback_len", ctypes.c_uint32), ("eager_window", ctypes.c_uint32),
                 ("candidates", ctypes.c_uint32), ("sample_len", ctypes.c_uint64), ("best_gbs", ctypes.c_double),
                 ("paper_gbs", ctypes.c_double), ("hit_rate", ctypes.c_double), ("variant", ctypes.c_int32),
-                ("preresolve", ctypes.c_uint32), ("lookback_width", ctypes.c_uint32)]
+                ("preresolve", ctypes.c_uint32), ("lookback_width", ctypes.c_uint32), ("chunk_bytes", ctypes.c_uint32)]
 
 
 class fsm_stats(ctypes.Structure):

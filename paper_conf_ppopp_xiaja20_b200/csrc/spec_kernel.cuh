@@ -48,8 +48,12 @@ __global__ void __launch_bounds__(kSpecThreads) spec_kernel(Params p, uint16_t *
                     cur[q0][i] = tb.init((uint32_t)__ldg(p.lb + c0 * KMAX + ((uint32_t)ii < ni ? ii : 0)));
                     acc[q0][i] = accf[q0][i] = 0;
                 }
+            // the next window block is in flight while this one is stepped (one HBM latency per
+            // window instead of one per 32 bytes)
+            Bytes32 xn = ldg256(p.in + b - Lw);
             for (uint32_t o = 0; o < Lw; o += 32) {
-                const Bytes32 x = ldg256(p.in + b - Lw + o);
+                const Bytes32 x = xn;
+                if (o + 32 < Lw) xn = ldg256(p.in + b - Lw + o + 32);
 #pragma unroll
                 for (int q = 0; q < 8; q++) {
 #pragma unroll

@@ -274,7 +274,7 @@ int fsm_compose_from(const fsm_shard_map *maps, uint32_t n, uint32_t start_state
  *   input, len   device pointer and length (symbols) of the input the runs will process
  *   k_min, k_max smallest / largest k to consider (0 = 1 / min(FSM_KMAX, n_states); k_min = k_max
  *                tunes only the windows for that k)
- *   sample_len   symbols timed per candidate (0 = min(len, 2 GiB)); the prefix is used, run with the
+ *   sample_len   symbols timed per candidate (0 = min(len, 4 GiB)); the prefix is used, run with the
  *                chunk and tile geometry of the full length so its cost per byte is the full run's
  *   out          the choice and its evidence; the chosen lookback_len / eager_window / variant are
  *                also written into the handle's options (the caller passes out->k to the runs)
